@@ -1,0 +1,160 @@
+"""CPU oracle for vbatched DPOTRF — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package. The product package
+(``paper_conf_ipps_abdelfattahhtd16_b200``) never imports it and shares no code with it.
+
+Thin ctypes wrapper over ``oracle/liboracle.so`` (built from ``oracle/oracle.c`` by
+``__graft_entry__.build()``); see ``oracle.c`` for the paper passages each routine follows,
+plus the numpy-only helpers used by the parity gates (row-scaled difference, SURVEY.md
+§8(c) reading #14). Parity status of every function is recorded in DESIGN.md §3.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liboracle.so")
+SRC_PATH = os.path.join(_HERE, "oracle.c")
+
+_dp = ctypes.POINTER(ctypes.c_double)
+_ip = ctypes.POINTER(ctypes.c_int)
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so (no FMA contraction, no fast-math, OpenMP)."""
+    if force or not os.path.exists(LIB_PATH) or os.path.getmtime(LIB_PATH) < os.path.getmtime(SRC_PATH):
+        cmd = ["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC",
+               "-o", LIB_PATH, SRC_PATH, "-lm"]
+        subprocess.check_call(cmd)
+    return LIB_PATH
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(LIB_PATH)
+        L.oracle_dpotrf_lower.argtypes = [ctypes.c_int, _dp, ctypes.c_int]
+        L.oracle_dpotrf_lower.restype = ctypes.c_int
+        L.oracle_dpotrf_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip, _ip, ctypes.c_int]
+        L.oracle_dpotrf_batch.restype = None
+        L.oracle_max_threads.argtypes = []
+        L.oracle_max_threads.restype = ctypes.c_int
+        L.oracle_dgemm.argtypes = [ctypes.c_char, ctypes.c_char, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                   ctypes.c_double, _dp, ctypes.c_int, _dp, ctypes.c_int, ctypes.c_double,
+                                   _dp, ctypes.c_int]
+        L.oracle_dsyrk.argtypes = [ctypes.c_char, ctypes.c_char, ctypes.c_int, ctypes.c_int, ctypes.c_double,
+                                   _dp, ctypes.c_int, ctypes.c_double, _dp, ctypes.c_int]
+        L.oracle_dtrsm.argtypes = [ctypes.c_char, ctypes.c_char, ctypes.c_char, ctypes.c_char, ctypes.c_int,
+                                   ctypes.c_int, ctypes.c_double, _dp, ctypes.c_int, _dp, ctypes.c_int]
+        L.oracle_backward_error.argtypes = [ctypes.c_int, _dp, ctypes.c_int, _dp, ctypes.c_int, ctypes.c_int]
+        L.oracle_backward_error.restype = ctypes.c_double
+        L.oracle_backward_error_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip,
+                                                  ctypes.POINTER(_dp), _ip, _ip, _dp, ctypes.c_int]
+        _lib = L
+    return _lib
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(_dp)
+
+
+def _fortran_block(a: np.ndarray) -> tuple[np.ndarray, int]:
+    """Return (array, ld) for a Fortran-ordered 2-D float64 array (a view, not a copy)."""
+    assert a.dtype == np.float64 and a.ndim == 2
+    if not a.flags.f_contiguous:
+        raise ValueError("expected a Fortran-ordered float64 array")
+    return a, max(1, a.shape[0])
+
+
+def dpotrf(a: np.ndarray) -> tuple[np.ndarray, int]:
+    """Oracle Cholesky of one matrix. `a` is n x n (only its lower triangle is read).
+    Returns (copy of a with L in the lower triangle, info)."""
+    out = np.array(a, dtype=np.float64, order="F", copy=True)
+    n = out.shape[0]
+    assert out.shape == (n, n)
+    info = lib().oracle_dpotrf_lower(n, _ptr(out), max(1, n))
+    return out, info
+
+
+def dpotrf_inplace(buf: np.ndarray, n: int, ld: int) -> int:
+    """Factor the n x n matrix stored column-major with leading dim ld in the flat float64
+    buffer `buf` (in place)."""
+    assert buf.dtype == np.float64 and buf.flags.c_contiguous
+    return lib().oracle_dpotrf_lower(n, _ptr(buf), ld)
+
+
+def dpotrf_batch(arena: np.ndarray, offsets, n, ld, nthreads: int = 0) -> np.ndarray:
+    """Factor a vbatched arena in place (OpenMP dynamic, one matrix per core).
+    arena: flat float64 array; offsets: element offsets of each matrix."""
+    n = np.ascontiguousarray(n, dtype=np.int32)
+    ld = np.ascontiguousarray(ld, dtype=np.int32)
+    B = len(n)
+    base = arena.ctypes.data
+    ptrs = (_dp * max(B, 1))(*[ctypes.cast(base + 8 * int(o), _dp) for o in offsets])
+    info = np.zeros(B, dtype=np.int32)
+    lib().oracle_dpotrf_batch(B, n.ctypes.data_as(_ip), ptrs, ld.ctypes.data_as(_ip),
+                              info.ctypes.data_as(_ip), int(nthreads))
+    return info
+
+
+def max_threads() -> int:
+    return lib().oracle_max_threads()
+
+
+def dgemm(ta, tb, alpha, A, B, beta, C):
+    C = np.array(C, dtype=np.float64, order="F", copy=True)
+    A = np.asfortranarray(A, dtype=np.float64)
+    B = np.asfortranarray(B, dtype=np.float64)
+    m, n = C.shape
+    k = A.shape[1] if ta == "N" else A.shape[0]
+    lib().oracle_dgemm(ta.encode(), tb.encode(), m, n, k, alpha, _ptr(A), max(1, A.shape[0]),
+                       _ptr(B), max(1, B.shape[0]), beta, _ptr(C), max(1, m))
+    return C
+
+
+def dsyrk(uplo, trans, alpha, A, beta, C):
+    C = np.array(C, dtype=np.float64, order="F", copy=True)
+    A = np.asfortranarray(A, dtype=np.float64)
+    n = C.shape[0]
+    k = A.shape[1] if trans == "N" else A.shape[0]
+    lib().oracle_dsyrk(uplo.encode(), trans.encode(), n, k, alpha, _ptr(A), max(1, A.shape[0]), beta,
+                       _ptr(C), max(1, n))
+    return C
+
+
+def dtrsm(side, uplo, transA, diag, alpha, A, B):
+    B = np.array(B, dtype=np.float64, order="F", copy=True)
+    A = np.asfortranarray(A, dtype=np.float64)
+    m, n = B.shape
+    lib().oracle_dtrsm(side.encode(), uplo.encode(), transA.encode(), diag.encode(), m, n, alpha,
+                       _ptr(A), max(1, A.shape[0]), _ptr(B), max(1, m))
+    return B
+
+
+def backward_error(A0: np.ndarray, L: np.ndarray, info: int) -> float:
+    """||A - L L^T||_F / (nb ||A||_F eps), eps = 2^-53, long double."""
+    A0 = np.asfortranarray(A0, dtype=np.float64)
+    L = np.asfortranarray(L, dtype=np.float64)
+    n = A0.shape[0]
+    return lib().oracle_backward_error(n, _ptr(A0), max(1, n), _ptr(L), max(1, L.shape[0]), int(info))
+
+
+def rowscaled_diff(Lg: np.ndarray, Lo: np.ndarray, nb: int) -> float:
+    """max_{i>=j} |Lg_ij - Lo_ij| / ||Lo(i, 0:i)||_2 over the leading nb x nb block
+    (SURVEY.md §8(c) reading #14)."""
+    if nb <= 0:
+        return 0.0
+    g = np.tril(np.asarray(Lg)[:nb, :nb])
+    o = np.tril(np.asarray(Lo)[:nb, :nb])
+    rn = np.sqrt(np.sum(o * o, axis=1))
+    rn[rn == 0] = 1.0
+    return float(np.max(np.abs(g - o) / rn[:, None]))

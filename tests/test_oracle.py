@@ -1,0 +1,363 @@
+"""Pins for the CPU oracle (oracle/oracle.c) against things the paper's problem and the
+mathematics fix — never against the oracle itself or the CUDA path (CPU only).
+
+PAPER.md prints no numeric worked example and no error bound (its figures are garbled),
+so the pins are (SURVEY.md §8(c) "What pins each part"):
+  closed forms (min(i,j), Pascal, hand-worked 2x2/3x3 golden fixtures), exact integer
+  families (integer unit-lower L, power-of-two diagonals), invariants (det, reconstruction),
+  library cross-checks (LAPACK dpotrf via MKL in torch; OpenBLAS via scipy), exact rational
+  Sylvester pivots on tiny integer matrices, and LAPACK info conventions.
+Each is chosen so a plausible oracle bug (dropped term, wrong sign/index, transposed
+operand, info off by one) fails at least one test.
+"""
+import json
+import math
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+import vbgen
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _chol(A):
+    return oracle.dpotrf(np.asfortranarray(np.asarray(A, dtype=np.float64)))
+
+
+# ---------------------------------------------------------------- golden / closed forms
+def test_handworked_golden():
+    g = json.load(open(os.path.join(GOLD, "handworked.json")))
+    for case in g["cases"]:
+        A = np.array(case["A"], dtype=np.float64)
+        L, info = _chol(A)
+        assert info == case["info"], case["name"]
+        if info == 0:
+            Lexp = np.array([[math.sqrt(2.0) if v == "sqrt2" else float(v) for v in row] for row in case["L"]])
+            assert np.array_equal(np.tril(L), Lexp), case["name"]  # bit-exact
+        else:
+            k = info - 1
+            lead = np.array(case["L_leading"], dtype=np.float64).reshape(k, k)
+            assert np.array_equal(np.tril(L[:k, :k]), lead), case["name"]
+            assert L[k, k] == case["pivot"], case["name"]  # LAPACK stores the failing pivot
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 7, 32, 33, 100, 200])
+def test_min_ij_gives_tril_ones(n):
+    i = np.arange(1, n + 1)
+    A = np.minimum.outer(i, i).astype(np.float64)
+    L, info = _chol(A)
+    assert info == 0
+    assert np.array_equal(np.tril(L), np.tril(np.ones((n, n))))
+
+
+@pytest.mark.parametrize("n", [1, 5, 12, 20, 29])
+def test_pascal_gives_lower_pascal(n):
+    P = np.array([[math.comb(i + j, j) for j in range(n)] for i in range(n)], dtype=np.float64)
+    Lp = np.array([[math.comb(i, j) if j <= i else 0 for j in range(n)] for i in range(n)], dtype=np.float64)
+    L, info = _chol(P)
+    assert info == 0
+    assert np.array_equal(np.tril(L), Lp)
+
+
+def _int_unit_lower(n, rng, diag=None):
+    L = np.tril(rng.integers(-1, 2, size=(n, n)), -1).astype(np.int64)
+    d = np.ones(n, dtype=np.int64) if diag is None else diag
+    L[np.arange(n), np.arange(n)] = d
+    return L
+
+
+@pytest.mark.parametrize("n", [2, 9, 33, 128])
+def test_integer_unit_lower_exact(n):
+    rng = np.random.default_rng(100 + n)
+    L = _int_unit_lower(n, rng)
+    A = (L @ L.T).astype(np.float64)  # exact: small integers
+    assert np.max(np.abs(L @ L.T)) < 2 ** 53
+    Lc, info = _chol(A)
+    assert info == 0
+    assert np.array_equal(np.tril(Lc), L.astype(np.float64))
+
+
+def test_integer_pow2_diagonal_exact():
+    rng = np.random.default_rng(7)
+    n = 64
+    L = _int_unit_lower(n, rng, diag=rng.choice([1, 2, 4], size=n))
+    A = (L @ L.T).astype(np.float64)
+    Lc, info = _chol(A)
+    assert info == 0
+    assert np.array_equal(np.tril(Lc), L.astype(np.float64))
+
+
+def test_identity_and_diagonal_and_scalar():
+    for n in (1, 4, 50):
+        L, info = _chol(np.eye(n))
+        assert info == 0 and np.array_equal(np.tril(L), np.eye(n))
+    d = 4.0 ** np.arange(10)
+    L, info = _chol(np.diag(d))
+    assert info == 0 and np.array_equal(np.tril(L), np.diag(2.0 ** np.arange(10)))
+    for a in (2.0, 3.0, 1e-300, 7.5e300):
+        L, info = _chol([[a]])
+        assert info == 0 and L[0, 0] == math.sqrt(a)
+
+
+def test_upper_triangle_never_read_or_written():
+    n = 40
+    A = vbgen.f1_matrix(9, 3, n)
+    ref, info_ref = _chol(A)
+    B = A.copy(order="F")
+    iu = np.triu_indices(n, 1)
+    B[iu] = np.nan
+    L, info = _chol(B)
+    assert info == info_ref == 0
+    assert np.array_equal(np.tril(L), np.tril(ref))
+    assert np.all(np.isnan(L[iu]))
+
+
+# ---------------------------------------------------------------- info conventions
+def test_info_special_cases():
+    assert _chol(np.ones((5, 5)))[1] == 2
+    assert _chol(np.zeros((3, 3)))[1] == 1
+    assert _chol([[-1.0]])[1] == 1
+    assert _chol(np.zeros((0, 0)))[1] == 0
+
+
+@pytest.mark.parametrize("n", [1, 2, 17, 64, 200])
+def test_info_negated_diagonal(n):
+    for gidx in range(0, 60, 7):
+        A = vbgen.f1_matrix(4, gidx, n, nonspd=True)
+        k = vbgen.nonspd_k(4, gidx, n)
+        L, info = _chol(A)
+        assert info == k
+        # leading block is the factor of the leading (k-1) block of A
+        if k > 1:
+            L2, info2 = _chol(A[: k - 1, : k - 1].copy(order="F"))
+            assert info2 == 0
+            assert np.array_equal(np.tril(L[: k - 1, : k - 1]), np.tril(L2))
+        assert L[k - 1, k - 1] < -n  # failing pivot stored (LAPACK dpotf2 convention)
+
+
+@pytest.mark.parametrize("pos", [(0, 0), (3, 3), (7, 7), (5, 2), (7, 0), (6, 5)])
+def test_info_nan_positions(pos):
+    """NaN at (k,k) -> info k+1; NaN at (i,j), i>j -> info i+1 (0-based positions);
+    matches MKL (LAPACK DISNAN semantics), SURVEY §8(c) reading #2."""
+    n = 8
+    A = vbgen.f1_matrix(1, 0, n)
+    i, j = pos
+    A[i, j] = np.nan
+    _, info = _chol(A)
+    assert info == i + 1
+
+
+def test_info_nan_matches_mkl():
+    import torch
+    n = 8
+    for (i, j) in [(2, 2), (3, 1), (7, 0)]:
+        A = vbgen.f1_matrix(1, 1, n)
+        A[i, j] = np.nan
+        A[j, i] = np.nan
+        _, info_m = torch.linalg.cholesky_ex(torch.from_numpy(A))
+        assert _chol(A)[1] == int(info_m)
+
+
+# ---------------------------------------------------------------- exact rationals (Sylvester)
+def _ldl_pivots(A):
+    """Exact rational pivots d_k = det(A_k)/det(A_{k-1}) by fraction-exact elimination."""
+    n = len(A)
+    M = [[Fraction(int(v)) for v in row] for row in A]
+    piv = []
+    for k in range(n):
+        d = M[k][k]
+        piv.append(d)
+        if d == 0:
+            break
+        for i in range(k + 1, n):
+            f = M[i][k] / d
+            for j in range(k, n):
+                M[i][j] -= f * M[k][j]
+    return piv
+
+
+def test_exact_rational_pivots_and_info():
+    rng = np.random.default_rng(11)
+    checked_fail = checked_ok = 0
+    for trial in range(300):
+        n = int(rng.integers(1, 11))
+        X = rng.integers(-3, 4, size=(n, n))
+        A = X @ X.T + np.diag(rng.integers(-6, 4, size=n))
+        A = (A + A.T) // 2
+        piv = _ldl_pivots(A)
+        k_exact = next((k + 1 for k, d in enumerate(piv) if d <= 0), 0)
+        # only judge cases where all float pivots are well separated from 0
+        if any(abs(float(d)) < 1e-6 for d in piv):
+            continue
+        L, info = _chol(A.astype(np.float64))
+        assert info == k_exact
+        nb = n if info == 0 else info - 1
+        for q in range(nb):
+            assert math.isclose(L[q, q] ** 2, float(piv[q]), rel_tol=1e-12)
+        checked_fail += info > 0
+        checked_ok += info == 0
+    assert checked_fail > 20 and checked_ok > 20
+
+
+# ---------------------------------------------------------------- invariants / library
+def test_det_invariant():
+    """prod l_jj^2 == det(A) with det from long-double partial-pivot LU (independent algorithm)."""
+    for n in (3, 10, 25):
+        A = vbgen.f1_matrix(2, n, n) / n
+        L, info = _chol(A)
+        assert info == 0
+        M = A.astype(np.longdouble).copy()
+        det = np.longdouble(1)
+        for k in range(n):
+            p = k + int(np.argmax(np.abs(M[k:, k])))
+            if p != k:
+                M[[k, p]] = M[[p, k]]
+                det = -det
+            det *= M[k, k]
+            M[k + 1:, k:] -= np.outer(M[k + 1:, k] / M[k, k], M[k, k:])
+        prod = np.prod(np.diag(L).astype(np.longdouble) ** 2)
+        assert abs(prod / det - 1) < 1e-12
+
+
+@pytest.mark.parametrize("n", [8, 64, 256])
+def test_random_well_conditioned_L_recovered(n):
+    rng = np.random.default_rng(n)
+    L = np.tril(rng.uniform(-1, 1, (n, n)) / n, -1) + np.diag(rng.uniform(1, 2, n))
+    A = np.asfortranarray(L @ L.T)
+    Lc, info = _chol(A)
+    assert info == 0
+    assert np.max(np.abs(np.tril(Lc) - L)) / np.max(np.abs(L)) < 1e-13
+
+
+@pytest.mark.parametrize("n", [1, 5, 40, 130, 300])
+def test_matches_mkl_dpotrf(n):
+    import torch
+    for gidx in range(3):
+        A = vbgen.f1_matrix(3, gidx, n)
+        L, info = _chol(A)
+        Lm, info_m = torch.linalg.cholesky_ex(torch.from_numpy(A))
+        assert info == int(info_m) == 0
+        assert oracle.rowscaled_diff(L, Lm.numpy(), n) < 1e-13
+        assert oracle.backward_error(A, L, info) < 1.0
+
+
+def test_matches_openblas_info_on_nonspd():
+    from scipy.linalg import lapack
+    for n in (5, 50, 120):
+        for gidx in (19, 39, 59):
+            A = vbgen.f1_matrix(4, gidx, n, nonspd=True)
+            _, info_s = lapack.dpotrf(A, lower=1, clean=0)
+            assert _chol(A)[1] == info_s
+
+
+def test_ill_conditioned_backward_error():
+    """F2 family: Q diag(lambda) Q^T with lambda log-uniform in [1,1e4]."""
+    rng = np.random.default_rng(5)
+    for n in (16, 64, 128):
+        Q, _ = np.linalg.qr(rng.standard_normal((n, n)))
+        lam = 10 ** rng.uniform(0, 4, n)
+        A = np.asfortranarray((Q * lam) @ Q.T)
+        A = np.asfortranarray((A + A.T) / 2)
+        L, info = _chol(A)
+        assert info == 0
+        assert oracle.backward_error(A, L, info) < 10
+
+
+def test_backward_error_detects_wrong_factor():
+    n = 20
+    A = vbgen.f1_matrix(1, 2, n)
+    L, info = _chol(A)
+    assert oracle.backward_error(A, L, info) < 10
+    L2 = L.copy(order="F")
+    L2[7, 3] *= (1 + 1e-10)
+    assert oracle.backward_error(A, L2, info) > 10
+
+
+def test_batch_equals_single():
+    n = np.array([0, 1, 5, 33, 64, 100, 2], dtype=np.int32)
+    ld = vbgen.ldda_for(n, "pad32")
+    off, tot = vbgen.arena_layout(n, ld)
+    arena = np.zeros(tot)
+    for b in range(len(n)):
+        A = vbgen.f1_matrix(1, b, int(n[b]), nonspd=(b == 3))
+        blk = np.zeros((ld[b], n[b]), order="F")
+        blk[: n[b], :] = A
+        arena[off[b]: off[b] + ld[b] * n[b]] = blk.ravel(order="F")
+    ref = arena.copy()
+    info = oracle.dpotrf_batch(arena, off, n, ld, nthreads=4)
+    for b in range(len(n)):
+        A = ref[off[b]: off[b] + ld[b] * n[b]].reshape((ld[b], n[b]), order="F")[: n[b]]
+        L1, i1 = _chol(np.asfortranarray(A))
+        got = arena[off[b]: off[b] + ld[b] * n[b]].reshape((ld[b], n[b]), order="F")[: n[b]]
+        assert info[b] == i1
+        assert np.array_equal(np.tril(got), np.tril(L1))
+    assert info[3] == vbgen.nonspd_k(1, 3, 33)
+
+
+# ---------------------------------------------------------------- BLAS oracles
+def _rand(rng, *shape):
+    return np.asfortranarray(rng.standard_normal(shape))
+
+
+@pytest.mark.parametrize("ta,tb", [("N", "N"), ("N", "T"), ("T", "N"), ("T", "T")])
+def test_gemm_oracle(ta, tb):
+    rng = np.random.default_rng(1)
+    m, n, k = 7, 5, 9
+    A = _rand(rng, m, k) if ta == "N" else _rand(rng, k, m)
+    B = _rand(rng, k, n) if tb == "N" else _rand(rng, n, k)
+    C = _rand(rng, m, n)
+    got = oracle.dgemm(ta, tb, 1.5, A, B, -0.5, C)
+    opA = A if ta == "N" else A.T
+    opB = B if tb == "N" else B.T
+    assert np.allclose(got, 1.5 * opA @ opB - 0.5 * C, rtol=1e-13, atol=1e-13)
+    # exact small-integer case
+    Ai = np.asfortranarray(rng.integers(-3, 4, A.shape).astype(float))
+    Bi = np.asfortranarray(rng.integers(-3, 4, B.shape).astype(float))
+    Ci = np.asfortranarray(rng.integers(-3, 4, C.shape).astype(float))
+    opA = Ai if ta == "N" else Ai.T
+    opB = Bi if tb == "N" else Bi.T
+    assert np.array_equal(oracle.dgemm(ta, tb, 1.0, Ai, Bi, 1.0, Ci), opA @ opB + Ci)
+
+
+@pytest.mark.parametrize("uplo,trans", [("L", "N"), ("L", "T"), ("U", "N"), ("U", "T")])
+def test_syrk_oracle(uplo, trans):
+    rng = np.random.default_rng(2)
+    n, k = 6, 4
+    A = _rand(rng, n, k) if trans == "N" else _rand(rng, k, n)
+    C = _rand(rng, n, n)
+    got = oracle.dsyrk(uplo, trans, -1.0, A, 1.0, C)
+    full = -(A @ A.T if trans == "N" else A.T @ A) + C
+    tri = np.tril if uplo == "L" else np.triu
+    other = np.triu if uplo == "L" else np.tril
+    assert np.allclose(tri(got), tri(full), rtol=1e-13, atol=1e-13)
+    assert np.array_equal(other(got, 1 if uplo == "L" else -1), other(C, 1 if uplo == "L" else -1))
+
+
+@pytest.mark.parametrize("side", ["L", "R"])
+@pytest.mark.parametrize("uplo", ["L", "U"])
+@pytest.mark.parametrize("ta", ["N", "T"])
+@pytest.mark.parametrize("diag", ["N", "U"])
+def test_trsm_oracle(side, uplo, ta, diag):
+    from scipy.linalg import solve_triangular
+    rng = np.random.default_rng(3)
+    m, n = 6, 5
+    na = m if side == "L" else n
+    A = _rand(rng, na, na) + 4 * np.eye(na)
+    A = np.asfortranarray(A)
+    B = _rand(rng, m, n)
+    X = oracle.dtrsm(side, uplo, ta, diag, 2.0, A, B)
+    T = np.tril(A) if uplo == "L" else np.triu(A)
+    if diag == "U":
+        np.fill_diagonal(T, 1.0)
+    opT = T if ta == "N" else T.T
+    if side == "L":
+        ref = solve_triangular(opT, 2.0 * B, lower=np.allclose(opT, np.tril(opT)))
+        assert np.allclose(opT @ X, 2.0 * B, rtol=1e-12, atol=1e-12)
+    else:
+        ref = solve_triangular(opT.T, (2.0 * B).T, lower=np.allclose(opT.T, np.tril(opT.T))).T
+        assert np.allclose(X @ opT, 2.0 * B, rtol=1e-12, atol=1e-12)
+    assert np.allclose(X, ref, rtol=1e-12, atol=1e-12)

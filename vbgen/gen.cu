@@ -1,0 +1,71 @@
+// vbgen device twin: fills a vbatched arena with the F1 family (see vbgen/__init__.py).
+// Holds none of the method's arithmetic; integer hash + one double add per diagonal entry,
+// bit-identical to the numpy version (pinned by tests/test_generator.py).
+//
+// Exported (C ABI, libvbgen.so):
+//   int vbgen_fill_f1(uint64_t seed, int batch, const int* d_n, const int* d_ldda,
+//                     double* const* d_A, const int* d_gidx, int nonspd_mod, int poison,
+//                     cudaStream_t stream)
+//     d_n/d_ldda/d_A/d_gidx: device arrays of length batch (d_gidx may be NULL -> gidx = i).
+//     Writes the lower triangle (and, if poison != 0, NaN-payload sentinels into the strict
+//     upper triangle and the padding rows n..ldda-1). Returns a cudaError_t.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace {
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
+  uint64_t z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+constexpr uint64_t kPoison = 0x7FF8DEADBEEF0001ull;
+
+// One CTA per matrix (grid-stride over matrices); threads stride over columns' rows.
+__global__ void fill_f1_kernel(uint64_t seed, int batch, const int* __restrict__ d_n,
+                               const int* __restrict__ d_ldda, double* const* __restrict__ d_A,
+                               const int* __restrict__ d_gidx, int nonspd_mod, int poison) {
+  const uint64_t s0 = splitmix64(seed);
+  for (int b = blockIdx.x; b < batch; b += gridDim.x) {
+    const int n = d_n[b];
+    if (n <= 0) continue;
+    const int ld = d_ldda[b];
+    const uint64_t g = d_gidx ? (uint64_t)d_gidx[b] : (uint64_t)b;
+    double* A = d_A[b];
+    int kneg = -1;
+    if (nonspd_mod > 0 && (int)(g % (uint64_t)nonspd_mod) == nonspd_mod - 1)
+      kneg = (int)(splitmix64(s0 ^ g ^ 0x5EEDull) % (uint64_t)n);
+    const int rows = poison ? ld : n;
+    for (int j = 0; j < n; ++j) {
+      double* col = A + (size_t)j * ld;
+      for (int i = (poison ? 0 : j) + threadIdx.x; i < rows; i += blockDim.x) {
+        double v;
+        if (i >= j && i < n) {
+          const uint64_t key = (g << 42) ^ ((uint64_t)i << 21) ^ (uint64_t)j;
+          v = (double)(splitmix64(s0 ^ key) >> 11) * 0x1.0p-53;
+          if (i == j) {
+            v = v + (double)n;
+            if (i == kneg) v = -v;
+          }
+        } else {
+          v = __longlong_as_double((long long)kPoison);
+        }
+        col[i] = v;
+      }
+    }
+  }
+}
+
+}  // namespace
+
+extern "C" int vbgen_fill_f1(uint64_t seed, int batch, const int* d_n, const int* d_ldda,
+                             double* const* d_A, const int* d_gidx, int nonspd_mod, int poison,
+                             cudaStream_t stream) {
+  if (batch <= 0) return 0;
+  int grid = batch < 148 * 16 ? batch : 148 * 16;
+  fill_f1_kernel<<<grid, 256, 0, stream>>>(seed, batch, d_n, d_ldda, d_A, d_gidx, nonspd_mod,
+                                           poison);
+  return (int)cudaGetLastError();
+}
