@@ -1,0 +1,92 @@
+"""Test/bench harness: builds vbatched device batches from vbgen recipes and compares
+results with the oracle. Infrastructure only (imports oracle lazily for the comparison
+helpers; the product package never imports this module)."""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+import vbgen
+from vbgen import device as vbdev
+
+
+class DeviceBatch:
+    """A vbatched problem resident in HBM: one arena (each matrix 256 B aligned), device
+    pointer array, n[], ldda[], info[] (int32), gidx[] (global matrix index for the hash)."""
+
+    def __init__(self, n, ldda=None, seed=1, gidx=None, nonspd_mod=0, device="cuda",
+                 ldda_mode="pad32"):
+        self.n = np.ascontiguousarray(n, dtype=np.int32)
+        self.B = len(self.n)
+        self.ldda = np.ascontiguousarray(vbgen.ldda_for(self.n, ldda_mode) if ldda is None else ldda,
+                                         dtype=np.int32)
+        self.gidx = np.arange(self.B, dtype=np.int32) if gidx is None else np.ascontiguousarray(gidx, np.int32)
+        self.seed = seed
+        self.nonspd_mod = nonspd_mod
+        self.device = torch.device(device)
+        self.off, total = vbgen.arena_layout(np.maximum(self.n, 0), self.ldda)
+        self.arena = torch.empty(total, dtype=torch.float64, device=self.device)
+        base = self.arena.data_ptr()
+        self.ptrs_h = (base + 8 * self.off).astype(np.int64)
+        self.d_ptrs = torch.from_numpy(self.ptrs_h).to(self.device)
+        self.d_n = torch.from_numpy(self.n).to(self.device)
+        self.d_ldda = torch.from_numpy(self.ldda).to(self.device)
+        self.d_gidx = torch.from_numpy(self.gidx).to(self.device)
+        self.d_info = torch.full((max(self.B, 1),), -12345, dtype=torch.int32, device=self.device)
+
+    def fill(self, poison=False, stream=None):
+        s = torch.cuda.current_stream().cuda_stream if stream is None else stream
+        vbdev.fill_f1(self.seed, self.B, self.d_n.data_ptr(), self.d_ldda.data_ptr(),
+                      self.d_ptrs.data_ptr(), self.d_gidx.data_ptr(), self.nonspd_mod, poison, s)
+        return self
+
+    def set_matrix(self, i, A: np.ndarray, poison=True):
+        """Write a host matrix (full n x n; only what the ldda block holds) into slot i."""
+        n, ld = int(self.n[i]), int(self.ldda[i])
+        blk = np.full((ld, n), np.nan)
+        if poison:
+            blk.view(np.uint64)[:] = np.uint64(vbgen.NAN_POISON_BITS)
+        blk[:n, :n] = np.where(np.tril(np.ones((n, n), bool)), A, blk[:n, :n])
+        t = torch.from_numpy(blk.ravel(order="F").copy())
+        self.arena[self.off[i]: self.off[i] + ld * n].copy_(t)
+
+    def block(self, i) -> np.ndarray:
+        """Host copy of the full ldda x n column block of matrix i."""
+        n, ld = int(self.n[i]), int(self.ldda[i])
+        if n <= 0:
+            return np.zeros((ld, 0))
+        return self.arena[self.off[i]: self.off[i] + ld * n].cpu().numpy().reshape((ld, n), order="F")
+
+    def host_arena(self) -> np.ndarray:
+        return self.arena.cpu().numpy()
+
+    def info(self) -> np.ndarray:
+        return self.d_info[: self.B].cpu().numpy()
+
+    def dpotrf(self, max_n=None, stream=None, uplo="L", check=True):
+        from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
+        mx = int(self.n.max()) if (max_n is None and self.B) else (max_n or 0)
+        return vbatched_dpotrf(uplo, self.d_n, self.d_ptrs, self.d_ldda, self.d_info, self.B, mx,
+                               stream=stream, check=check)
+
+    def host_matrix_input(self, i) -> np.ndarray:
+        """The matrix the generator writes for slot i (numpy twin)."""
+        return vbgen.f1_matrix(self.seed, int(self.gidx[i]), int(self.n[i]),
+                               self.nonspd_mod > 0 and int(self.gidx[i]) % self.nonspd_mod == self.nonspd_mod - 1)
+
+
+def compare_with_oracle(A_in: np.ndarray, L_gpu: np.ndarray, info_gpu: int, kappa_ok=True):
+    """Parity gates (BASELINE.json north_star):
+    info bit-exact; backward error <= 10 (eps = 2^-53) on the defined leading block;
+    row-scaled difference to the oracle's L <= 1e-10. Returns dict of measurements."""
+    import oracle
+    n = A_in.shape[0]
+    Lo, info_o = oracle.dpotrf(np.asfortranarray(A_in))
+    res = {"n": n, "info_oracle": info_o, "info_gpu": int(info_gpu)}
+    nb = n if info_o == 0 else info_o - 1
+    Lg = np.asfortranarray(L_gpu[:n, :n])
+    res["bwd"] = oracle.backward_error(np.asfortranarray(A_in), Lg, info_o) if nb > 0 else 0.0
+    res["rowscaled"] = oracle.rowscaled_diff(Lg, Lo, nb)
+    res["ok"] = (res["info_oracle"] == res["info_gpu"] and res["bwd"] <= 10.0 and
+                 (res["rowscaled"] <= 1e-10 or not kappa_ok))
+    return res

@@ -1,0 +1,139 @@
+/*
+ * vbatched.h — C ABI of the B200-native variable-size batched Cholesky library
+ * (libvbatched.so, built from paper_conf_ipps_abdelfattahhtd16_b200/csrc/).
+ *
+ * Problem (Fig. 1; §III-A): a batch of k independent
+ * dense matrices, matrix i being N_i x N_i with its own leading dimension LDA_i, each
+ * factored as A_i = L_i L_i^T. A "vbatched" routine takes an array of pointers, the arrays
+ * of sizes and leading dimensions (resident in GPU memory) and the batch
+ * count; the max-given interface additionally takes the maximum size
+ * (PAPER.md:388-412), the LAPACK-like one computes it on the GPU.
+ *
+ * Conventions for every routine below
+ *  - Matrices are column-major doubles: element (r,c) of matrix i is dA_array[i][r + c*ldda[i]].
+ *  - Pointer arguments prefixed d are DEVICE pointers on the current CUDA device; h = host.
+ *    The caller owns every array; the library never frees or reallocates caller memory.
+ *  - All int arguments are 32-bit. Offsets inside the library are computed in 64 bits.
+ *  - Asynchronous: work is enqueued on `stream` (0 = legacy default stream); no host
+ *    synchronisation and no device->host copy happens unless the routine says so. Internal
+ *    workspace (O(batchCount) ints) is stream-ordered (cudaMallocAsync/cudaFreeAsync).
+ *  - Return value: 0 = enqueued; -p = host-scalar argument number p (1-based) is invalid,
+ *    nothing enqueued; > 0 = a cudaError_t from the launch.
+ *  - batchCount == 0 returns 0 and enqueues nothing.
+ *  - No CPU fallback exists: every arithmetic step runs in this library's CUDA kernels
+ *    (sm_100a). If no device is present the call returns the CUDA error.
+ */
+#ifndef VBATCHED_H_
+#define VBATCHED_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* vb_stream_t; /* == cudaStream_t */
+
+/* ---------------------------------------------------------------------------------------
+ * vbatched_dpotrf — FP64 variable-size batched Cholesky, max-given interface.
+ * Cite: PAPER.md:520-549 (§III-D, Algorithm 1: panel update (syrk) -> tile factorize (potf2)
+ * -> panel factorize (trsm)); PAPER.md:724-812 (§III-E separated kernels); error reporting
+ * follows LAPACK DPOTRF [7] (PAPER.md:2291-2297 lists it as future work).
+ *
+ *  uplo       'L' (lower) — the factor L overwrites the lower triangle of each A_i.
+ *             'U' is not yet supported and returns -1.
+ *  d_n        [batchCount] matrix orders n_i (device).
+ *  dA_array   [batchCount] device pointers to the matrices (device array of device ptrs).
+ *  d_ldda     [batchCount] leading dimensions (device); must be >= max(1, n_i).
+ *  d_info     [batchCount] output (device), LAPACK semantics per matrix:
+ *               0  success;
+ *               k>0 the leading minor of order k is not positive definite: the k-th pivot
+ *                  was <= 0 or NaN. Columns 1..k-1 hold L of the leading block; the failing
+ *                  pivot value is stored at (k,k); the rest of the lower triangle is
+ *                  implementation-defined (partially updated).
+ *              -2  n_i < 0;  -4  ldda_i < max(1,n_i);  -7  n_i > max_n.  (matrix untouched)
+ *  batchCount number of matrices (>= 0)                                      (-6 if < 0)
+ *  max_n      an upper bound on every n_i (host)                              (-7 if < 0)
+ *  stream     CUDA stream.
+ * The strict upper triangle and rows n_i..ldda_i-1 are never read nor written.
+ * Matrices must not overlap. Returns 0 / -p / cudaError_t as described above.
+ */
+int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream);
+
+/* LAPACK-like interface: identical to vbatched_dpotrf but max_n is not
+ * needed; the device scan computes it (no host synchronisation: launch sizes assume the
+ * worst case and idle CTAs exit). Argument numbers as above; there is no check -7. */
+int vbatched_dpotrf_nomax(char uplo, const int* d_n, double* const* dA_array,
+                          const int* d_ldda, int* d_info, int batchCount, vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
+ * vbatched_dpotrf_host — end-to-end variant on HOST memory (blocking).
+ * Same problem and semantics as vbatched_dpotrf, but h_n, hA_array (host pointers to host
+ * matrices, ideally pinned), h_ldda and h_info live in host memory. The library streams the
+ * batch through a device staging ring in chunks: H2D copy of a chunk's matrices, factor
+ * (the same kernels as vbatched_dpotrf), D2H copy back, with copies of neighbouring chunks
+ * overlapping the factorisation. Each matrix's whole ldda x n column block is copied in
+ * and back (the strict upper triangle and padding rows are returned unchanged).
+ * Returns when every result is back in host memory. workspace_bytes bounds the device
+ * staging memory (0 = library default, 4 GiB). Argument checks as vbatched_dpotrf
+ * (-2 n<0 and -4 ldda<max(1,n) are reported in h_info, -7 if n > max_n).
+ * Extra return code: -9 = workspace_bytes too small for the largest matrix. */
+int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA_array, const int* h_ldda,
+                         int* h_info, int batchCount, int max_n, size_t workspace_bytes,
+                         vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
+ * vbatched BLAS used by the blocked factorisation (§III-E.2/3), exposed
+ * as standalone entry points. Per-matrix dimension arrays are device arrays; dimensions are
+ * assumed valid (MAGMA "_nocheck" convention); host scalars are checked.
+ *
+ * vbatched_dgemm: C_i = alpha op(A_i) op(B_i) + beta C_i, C_i m_i x n_i, op(A_i) m_i x k_i.
+ *   transA, transB in {'N','T'} (args 1,2). max_m/max_n/max_k >= every m_i/n_i/k_i
+ *   (args 16-18; -p if < 0). beta == 0 does not read C. (DMMA tensor-core kernel.)
+ */
+int vbatched_dgemm(char transA, char transB, const int* d_m, const int* d_n, const int* d_k,
+                   double alpha, const double* const* dA_array, const int* d_ldda,
+                   const double* const* dB_array, const int* d_lddb, double beta,
+                   double* const* dC_array, const int* d_lddc, int batchCount, int max_m,
+                   int max_n, int max_k, vb_stream_t stream);
+
+/* vbatched_dsyrk: C_i = alpha A_i A_i^T + beta C_i (trans 'N', A_i n_i x k_i) or
+ *   alpha A_i^T A_i + beta C_i (trans 'T', A_i k_i x n_i), only the `uplo` triangle of C_i
+ *   is referenced/updated. uplo in {'L','U'} (arg 1), trans in {'N','T'} (arg 2). */
+int vbatched_dsyrk(char uplo, char trans, const int* d_n, const int* d_k, double alpha,
+                   const double* const* dA_array, const int* d_ldda, double beta,
+                   double* const* dC_array, const int* d_lddc, int batchCount, int max_n,
+                   int max_k, vb_stream_t stream);
+
+/* vbatched_dtrsm: solve op(A_i) X = alpha B_i (side 'L') or X op(A_i) = alpha B_i (side 'R'),
+ *   X overwriting B_i (m_i x n_i); A_i triangular (uplo 'L'/'U'), op = transA ('N'/'T'),
+ *   diag 'N' or 'U' (unit). Cholesky uses side 'R', uplo 'L', transA 'T', diag 'N'
+ *   ("C2 = C2 C1^-T"). Implemented as an in-shared-memory inversion of the
+ *   diagonal blocks (TRTRI) followed by DMMA GEMMs, the design PAPER.md:760-772 describes.
+ *   Supported now: side 'R' with any uplo/transA/diag; side 'L' returns -1 (NEXT-2). */
+int vbatched_dtrsm(char side, char uplo, char transA, char diag, const int* d_m, const int* d_n,
+                   double alpha, const double* const* dA_array, const int* d_ldda,
+                   double* const* dB_array, const int* d_lddb, int batchCount, int max_m,
+                   int max_n, vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Host helpers (pure host, deterministic, no CUDA).
+ * vbatched_partition_lpt: flop-balanced multi-GPU sharding: longest
+ *   processing time first on cost n^3/3 — sort by n descending (ties by index), assign
+ *   each matrix to the least-loaded rank (ties to the lowest rank). h_owner[i] in [0,ngpu).
+ *   Returns 0, or -2 (batchCount < 0), -3 (ngpu < 1). */
+int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owner);
+
+/* Library version string and the tuning constants compiled in (for logs). */
+const char* vbatched_version(void);
+
+/* Pinned host memory helpers (cudaHostAlloc / cudaFreeHost) for the _host entry point. */
+void* vbatched_host_alloc(size_t bytes);
+int vbatched_host_free(void* p);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* VBATCHED_H_ */

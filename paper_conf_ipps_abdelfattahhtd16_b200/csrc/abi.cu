@@ -1,0 +1,153 @@
+// abi.cu — the C ABI of libvbatched.so (declared and documented in include/vbatched.h).
+// Host-side work is O(1) per call (argument checks, workspace, launches) except for the
+// host-buffer streaming entry point and the pure-host partition helper.
+#include <algorithm>
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "../../include/vbatched.h"
+#include "common.cuh"
+#include "internal.h"
+
+namespace vb {
+
+static bool g_pool_configured = false;
+
+cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream) {
+  if (!g_pool_configured) {
+    // Keep freed workspace in the device's default pool (no OS round trip per call).
+    int dev;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = 256ull << 20;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    g_pool_configured = true;
+  }
+  return cudaMallocAsync(p, bytes, stream);
+}
+
+cudaError_t ws_free(void* p, cudaStream_t stream) { return cudaFreeAsync(p, stream); }
+
+static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                      int batch, int max_n, bool check_max, cudaStream_t stream) {
+  if (uplo != 'L' && uplo != 'l') return -1;  // 'U' is NEXT-1 (include/vbatched.h)
+  if (batch < 0) return -6;
+  if (check_max && max_n < 0) return -7;
+  if (batch == 0) return 0;
+  void* ws = nullptr;
+  const size_t bytes = sizeof(Ctrl) + sizeof(int) * (size_t)batch;
+  cudaError_t e = ws_alloc(&ws, bytes, stream);
+  if (e != cudaSuccess) return (int)e;
+  Ctrl* ctrl = static_cast<Ctrl*>(ws);
+  int* order = reinterpret_cast<int*>(ctrl + 1);
+  e = launch_scan_bin(d_n, d_ldda, d_info, batch, max_n, check_max, ctrl, order, stream);
+  if (e == cudaSuccess) {
+    const int hint = check_max ? max_n : (1 << 30);
+    if (hint > 0) e = launch_potrf_paths(d_n, dA, d_ldda, d_info, batch, hint, ctrl, order, stream);
+  }
+  cudaError_t e2 = ws_free(ws, stream);
+  if (e == cudaSuccess) e = e2;
+  return (int)e;
+}
+
+}  // namespace vb
+
+using namespace vb;
+
+extern "C" {
+
+int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream) {
+  return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, max_n, true,
+                    (cudaStream_t)stream);
+}
+
+int vbatched_dpotrf_nomax(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
+                          int* d_info, int batchCount, vb_stream_t stream) {
+  return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, 0, false,
+                    (cudaStream_t)stream);
+}
+
+int vbatched_dgemm(char transA, char transB, const int* d_m, const int* d_n, const int* d_k,
+                   double alpha, const double* const* dA_array, const int* d_ldda,
+                   const double* const* dB_array, const int* d_lddb, double beta,
+                   double* const* dC_array, const int* d_lddc, int batchCount, int max_m,
+                   int max_n, int max_k, vb_stream_t stream) {
+  auto okT = [](char t) { return t == 'N' || t == 'n' || t == 'T' || t == 't' || t == 'C' || t == 'c'; };
+  if (!okT(transA)) return -1;
+  if (!okT(transB)) return -2;
+  if (batchCount < 0) return -14;
+  if (max_m < 0) return -15;
+  if (max_n < 0) return -16;
+  if (max_k < 0) return -17;
+  if (batchCount == 0) return 0;
+  return gemm_launch(transA, transB, d_m, d_n, d_k, alpha, dA_array, d_ldda, dB_array, d_lddb, beta,
+                     dC_array, d_lddc, batchCount, max_m, max_n, max_k, (cudaStream_t)stream);
+}
+
+int vbatched_dsyrk(char uplo, char trans, const int* d_n, const int* d_k, double alpha,
+                   const double* const* dA_array, const int* d_ldda, double beta,
+                   double* const* dC_array, const int* d_lddc, int batchCount, int max_n,
+                   int max_k, vb_stream_t stream) {
+  if (!(uplo == 'L' || uplo == 'l' || uplo == 'U' || uplo == 'u')) return -1;
+  if (!(trans == 'N' || trans == 'n' || trans == 'T' || trans == 't' || trans == 'C' || trans == 'c')) return -2;
+  if (batchCount < 0) return -11;
+  if (max_n < 0) return -12;
+  if (max_k < 0) return -13;
+  if (batchCount == 0) return 0;
+  return syrk_launch(uplo, trans, d_n, d_k, alpha, dA_array, d_ldda, beta, dC_array, d_lddc,
+                     batchCount, max_n, max_k, (cudaStream_t)stream);
+}
+
+int vbatched_dtrsm(char side, char uplo, char transA, char diag, const int* d_m, const int* d_n,
+                   double alpha, const double* const* dA_array, const int* d_ldda,
+                   double* const* dB_array, const int* d_lddb, int batchCount, int max_m,
+                   int max_n, vb_stream_t stream) {
+  if (!(side == 'R' || side == 'r')) return -1;  // side 'L' is NEXT-2
+  if (!(uplo == 'L' || uplo == 'l' || uplo == 'U' || uplo == 'u')) return -2;
+  if (!(transA == 'N' || transA == 'n' || transA == 'T' || transA == 't' || transA == 'C' || transA == 'c')) return -3;
+  if (!(diag == 'N' || diag == 'n' || diag == 'U' || diag == 'u')) return -4;
+  if (batchCount < 0) return -12;
+  if (max_m < 0) return -13;
+  if (max_n < 0) return -14;
+  if (batchCount == 0) return 0;
+  return trsm_launch(side, uplo, transA, diag, d_m, d_n, alpha, dA_array, d_ldda, dB_array, d_lddb,
+                     batchCount, max_m, max_n, (cudaStream_t)stream);
+}
+
+int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owner) {
+  if (batchCount < 0) return -2;
+  if (ngpu < 1) return -3;
+  std::vector<int> idx(batchCount);
+  std::iota(idx.begin(), idx.end(), 0);
+  std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return h_n[a] > h_n[b]; });
+  std::vector<double> load(ngpu, 0.0);
+  for (int i : idx) {
+    int best = 0;
+    for (int r = 1; r < ngpu; ++r)
+      if (load[r] < load[best]) best = r;
+    const double n = h_n[i] > 0 ? (double)h_n[i] : 0.0;
+    load[best] += n * n * n / 3.0;
+    h_owner[i] = best;
+  }
+  return 0;
+}
+
+const char* vbatched_version(void) {
+  return "libvbatched 0.1 (sm_100a; blocked NB=32 MB=128 KC=16 stages=3; warp path n<=32; "
+         "DMMA m8n8k4 f64)";
+}
+
+void* vbatched_host_alloc(size_t bytes) {
+  void* p = nullptr;
+  if (cudaHostAlloc(&p, bytes, cudaHostAllocDefault) != cudaSuccess) return nullptr;
+  return p;
+}
+
+int vbatched_host_free(void* p) { return (int)cudaFreeHost(p); }
+
+}  // extern "C"

@@ -1,0 +1,466 @@
+// blas.cu — standalone vbatched DGEMM / DSYRK / DTRSM (§III-E.2-3) on the
+// FP64 tensor cores (DMMA m8n8k4), exposed through include/vbatched.h.
+//
+// Work distribution (replaces the paper's max-size grid with early-exit thread blocks,
+// PAPER.md:633-674, which is Kepler prior art): a one-CTA device scan turns the per-matrix
+// dimensions into a prefix sum of tile counts; persistent CTAs then pop global tile ids from
+// an atomic counter and locate their matrix by binary search. Only real tiles are visited —
+// for SYRK only the tiles of the referenced triangle ("decision layer").
+#include <algorithm>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace vb {
+namespace {
+
+constexpr int kBT = 64;      // C tile edge
+constexpr int kBK = 16;      // k chunk
+constexpr int kGThreads = 128;
+constexpr int kLD = kBT + 4;
+
+enum Mode { kGemm = 0, kSyrkLower = 1, kSyrkUpper = 2, kTrsm = 3 };
+
+struct BlasArgs {
+  int mode;
+  bool ta, tb;  // operand transposed
+  const int* m;
+  const int* n;
+  const int* k;
+  double alpha, beta;
+  const double* const* A;
+  const int* lda;
+  const double* const* B;
+  const int* ldb;
+  double* const* C;
+  const int* ldc;
+  int batch;
+  // trsm
+  bool tlower, unit, upper_in_A;
+};
+
+__device__ __forceinline__ int cdiv(int a, int b) { return (a + b - 1) / b; }
+
+__device__ __forceinline__ int tiles_of(const BlasArgs& a, int i) {
+  if (a.mode == kGemm) {
+    const int m = a.m[i], n = a.n[i];
+    return (m > 0 && n > 0) ? cdiv(m, kBT) * cdiv(n, kBT) : 0;
+  }
+  if (a.mode == kTrsm) {
+    const int m = a.m[i], n = a.n[i];
+    return (m > 0 && n > 0) ? cdiv(m, kBT) : 0;
+  }
+  const int n = a.n[i];
+  const int t = n > 0 ? cdiv(n, kBT) : 0;
+  return t * (t + 1) / 2;
+}
+
+// Prefix sum of tile counts (one CTA of 1024 threads, carry across 1024-wide chunks).
+__global__ void __launch_bounds__(1024, 1) tile_scan_kernel(BlasArgs a, int* off, int* counter) {
+  pdl_launch_dependents();
+  __shared__ int wsum[32];
+  __shared__ int carry;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) carry = 0;
+  __syncthreads();
+  for (int base = 0; base < a.batch; base += 1024) {
+    const int i = base + tid;
+    const int v = i < a.batch ? tiles_of(a, i) : 0;
+    int incl = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl += t;
+    }
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+      const int w = wsum[lane];
+      int x = w;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += t;
+      }
+      wsum[lane] = x - w;
+    }
+    __syncthreads();
+    const int c = carry;
+    if (i < a.batch) off[i] = c + wsum[warp] + incl - v;
+    __syncthreads();
+    if (tid == 1023) carry = c + wsum[warp] + incl;
+    __syncthreads();
+  }
+  if (tid == 0) {
+    off[a.batch] = carry;
+    *counter = 0;
+  }
+}
+
+__device__ __forceinline__ int find_matrix(const int* off, int batch, int t) {
+  int lo = 0, hi = batch;  // largest i with off[i] <= t and tiles > 0
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (off[mid] <= t) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// ---------------------------------------------------------------------------------------
+// GEMM / SYRK tile: C[r0:r0+64, c0:c0+64] = alpha op(A) op(B) + beta C (masked for SYRK).
+struct GemmSmem {
+  double a[2][kBK][kLD];  // [k][row]
+  double b[2][kBK][kLD];  // [k][col]
+};
+
+__device__ __forceinline__ void gemm_stage(GemmSmem& s, int st, const double* A, int lda, bool ta,
+                                           const double* B, int ldb, bool tb, int m, int n, int K,
+                                           int r0, int c0, int k0) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int e = 0; e < (kBT * kBK) / kGThreads; ++e) {
+    const int idx = tid + e * kGThreads;
+    int i, k;
+    if (!ta) { i = idx % kBT; k = idx / kBT; }
+    else { k = idx % kBK; i = idx / kBK; }
+    const bool p = (r0 + i < m) && (k0 + k < K);
+    const size_t o = !ta ? (size_t)(k0 + k) * lda + (r0 + i) : (size_t)(r0 + i) * lda + (k0 + k);
+    cp_async8(&s.a[st][k][i], A + (p ? o : 0), p);
+  }
+#pragma unroll
+  for (int e = 0; e < (kBT * kBK) / kGThreads; ++e) {
+    const int idx = tid + e * kGThreads;
+    int j, k;
+    if (!tb) { k = idx % kBK; j = idx / kBK; }
+    else { j = idx % kBT; k = idx / kBT; }
+    const bool p = (c0 + j < n) && (k0 + k < K);
+    const size_t o = !tb ? (size_t)(c0 + j) * ldb + (k0 + k) : (size_t)(k0 + k) * ldb + (c0 + j);
+    cp_async8(&s.b[st][k][j], B + (p ? o : 0), p);
+  }
+}
+
+__global__ void __launch_bounds__(kGThreads) gemm_syrk_kernel(BlasArgs a, const int* off,
+                                                              int* counter) {
+  __shared__ __align__(16) GemmSmem s;
+  __shared__ int s_t;
+  pdl_wait();
+  const int total = off[a.batch];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  const int wr = (warp >> 1) * 32, wc = (warp & 1) * 32;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(counter, 1);
+    __syncthreads();
+    const int t = s_t;
+    __syncthreads();
+    if (t >= total) break;
+    const int mi = find_matrix(off, a.batch, t);
+    int lt = t - off[mi];
+    const int n = a.n[mi];
+    const int m = (a.mode == kGemm) ? a.m[mi] : n;
+    const int K = a.k[mi];
+    int ti, tj;
+    if (a.mode == kGemm) {
+      const int tm = cdiv(m, kBT);
+      ti = lt % tm;
+      tj = lt / tm;
+    } else {
+      const int T = cdiv(n, kBT);
+      // enumerate the triangle column by column
+      int col = 0;
+      while (true) {
+        const int len = (a.mode == kSyrkLower) ? T - col : col + 1;
+        if (lt < len) break;
+        lt -= len;
+        ++col;
+      }
+      tj = col;
+      ti = (a.mode == kSyrkLower) ? col + lt : lt;
+    }
+    const int r0 = ti * kBT, c0 = tj * kBT;
+    const double* A = a.A[mi];
+    const double* B = (a.mode == kGemm) ? a.B[mi] : a.A[mi];
+    const int lda = a.lda[mi];
+    const int ldb = (a.mode == kGemm) ? a.ldb[mi] : lda;
+    double acc[4][4][2];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+      for (int y = 0; y < 4; ++y) acc[x][y][0] = acc[x][y][1] = 0.0;
+    const int nk = cdiv(K, kBK);
+    if (nk > 0) gemm_stage(s, 0, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, 0);
+    cp_async_commit();
+    for (int kc = 0; kc < nk; ++kc) {
+      if (kc + 1 < nk)
+        gemm_stage(s, (kc + 1) & 1, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, (kc + 1) * kBK);
+      cp_async_commit();
+      cp_async_wait<1>();
+      __syncthreads();
+      const int st = kc & 1;
+#pragma unroll
+      for (int kk = 0; kk < kBK / 4; ++kk) {
+        double fa[4], fb[4];
+#pragma unroll
+        for (int x = 0; x < 4; ++x) fa[x] = s.a[st][kk * 4 + q][wr + x * 8 + g];
+#pragma unroll
+        for (int y = 0; y < 4; ++y) fb[y] = s.b[st][kk * 4 + q][wc + y * 8 + g];
+#pragma unroll
+        for (int x = 0; x < 4; ++x)
+#pragma unroll
+          for (int y = 0; y < 4; ++y) dmma(acc[x][y], fa[x], fb[y]);
+      }
+      __syncthreads();
+    }
+    cp_async_wait<0>();
+    double* C = a.C[mi];
+    const int ldc = a.ldc[mi];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+      for (int y = 0; y < 4; ++y)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int r = r0 + wr + x * 8 + g, c = c0 + wc + y * 8 + 2 * q + h;
+          if (r >= m || c >= n) continue;
+          if (a.mode == kSyrkLower && r < c) continue;
+          if (a.mode == kSyrkUpper && r > c) continue;
+          double* pc = C + (size_t)c * ldc + r;
+          const double v = a.alpha * acc[x][y][h];
+          *pc = (a.beta == 0.0) ? v : fma(a.beta, *pc, v);
+        }
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// TRSM side 'R': X T = alpha B, T = op(A) (n x n triangular), one CTA per 64-row block of B.
+// Column blocks of 32 are solved in dependency order (ascending for upper T, descending for
+// lower T): R = alpha B_J - sum_K X_K T_{K,J} (DMMA), X_J = R inv(T_JJ) (TRTRI in smem + DMMA).
+constexpr int kTW = 32;
+struct TrsmSmem {
+  double x[kTW][kLD];     // A operand [k][row]
+  double t[kTW][kTW + 4];  // B operand [k][col]
+  double d[kTW][kTW + 1];  // raw diagonal block T_JJ [row][col]
+  double inv[kTW][kTW + 4];  // inv(T_JJ) [k][col]
+};
+
+__device__ __forceinline__ double t_elem(const BlasArgs& a, const double* A, int lda, int i, int j) {
+  // T(i,j) = op(A)(i,j) restricted to A's triangle; unit diagonal if requested.
+  if (i == j && a.unit) return 1.0;
+  const int ai = a.ta ? j : i, aj = a.ta ? i : j;
+  const bool in_tri = a.upper_in_A ? (ai <= aj) : (ai >= aj);
+  return in_tri ? A[(size_t)aj * lda + ai] : 0.0;
+}
+
+__global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* off, int* counter) {
+  __shared__ __align__(16) TrsmSmem s;
+  __shared__ int s_t;
+  pdl_wait();
+  const int total = off[a.batch];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  const int wr = (warp >> 1) * 32, wc = (warp & 1) * 16;
+  for (;;) {
+    if (tid == 0) s_t = atomicAdd(counter, 1);
+    __syncthreads();
+    const int t = s_t;
+    __syncthreads();
+    if (t >= total) break;
+    const int mi = find_matrix(off, a.batch, t);
+    const int r0 = (t - off[mi]) * kBT;
+    const int m = a.m[mi], n = a.n[mi];
+    const double* A = a.A[mi];
+    const int lda = a.lda[mi];
+    double* B = a.C[mi];
+    const int ldb = a.ldc[mi];
+    const int nbk = cdiv(n, kTW);
+    for (int step = 0; step < nbk; ++step) {
+      const int J = a.tlower ? nbk - 1 - step : step;
+      const int c0 = J * kTW, w = min(kTW, n - c0);
+      double acc[4][2][2];
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 2; ++y) acc[x][y][0] = acc[x][y][1] = 0.0;
+      // sum over solved blocks K of X_K T_{K,J}
+      for (int s2 = 0; s2 < step; ++s2) {
+        const int Kb = a.tlower ? nbk - 1 - s2 : s2;
+        const int k0 = Kb * kTW, kw = min(kTW, n - k0);
+        for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
+          const int k = idx / kBT, i = idx % kBT;
+          s.x[k][i] = (k < kw && r0 + i < m) ? B[(size_t)(k0 + k) * ldb + r0 + i] : 0.0;
+        }
+        for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
+          const int j = idx / kTW, k = idx % kTW;
+          s.t[k][j] = (k < kw && j < w) ? t_elem(a, A, lda, k0 + k, c0 + j) : 0.0;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k4 = 0; k4 < kTW / 4; ++k4) {
+          double fa[4], fb[2];
+#pragma unroll
+          for (int x = 0; x < 4; ++x) fa[x] = s.x[k4 * 4 + q][wr + x * 8 + g];
+#pragma unroll
+          for (int y = 0; y < 2; ++y) fb[y] = s.t[k4 * 4 + q][wc + y * 8 + g];
+#pragma unroll
+          for (int x = 0; x < 4; ++x)
+#pragma unroll
+            for (int y = 0; y < 2; ++y) dmma(acc[x][y], fa[x], fb[y]);
+        }
+        __syncthreads();
+      }
+      // R = alpha B_J - acc, into s.x as [k=col][row]; diagonal block into s.d
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 2; ++y)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) s.x[wc + y * 8 + 2 * q + h][wr + x * 8 + g] = -acc[x][y][h];
+      for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
+        const int j = idx / kTW, i = idx % kTW;
+        s.d[i][j] = (i < w && j < w) ? t_elem(a, A, lda, c0 + i, c0 + j) : (i == j ? 1.0 : 0.0);
+      }
+      __syncthreads();
+      for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
+        const int k = idx / kBT, i = idx % kBT;
+        const double bv = (k < w && r0 + i < m) ? B[(size_t)(c0 + k) * ldb + r0 + i] : 0.0;
+        s.x[k][i] = fma(a.alpha, bv, s.x[k][i]);
+      }
+      // inv(T_JJ): lane j of warp 0 computes column j by substitution
+      if (warp == 0) {
+        const int j = lane;
+        double xcol[kTW];
+        if (!a.tlower) {  // upper: x_i = 0 (i>j), x_j = 1/d_jj, x_i = -(sum_{k=i+1..j} d_ik x_k)/d_ii
+#pragma unroll
+          for (int i = kTW - 1; i >= 0; --i) {
+            double acc2 = 0.0;
+#pragma unroll
+            for (int k = i + 1; k < kTW; ++k) acc2 = fma(s.d[i][k], xcol[k], acc2);
+            const double r = 1.0 / s.d[i][i];
+            xcol[i] = (i > j) ? 0.0 : (i == j ? r : -acc2 * r);
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < kTW; ++i) {
+            double acc2 = 0.0;
+#pragma unroll
+            for (int k = 0; k < i; ++k) acc2 = fma(s.d[i][k], xcol[k], acc2);
+            const double r = 1.0 / s.d[i][i];
+            xcol[i] = (i < j) ? 0.0 : (i == j ? r : -acc2 * r);
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < kTW; ++i) s.inv[i][j] = xcol[i];
+      }
+      __syncthreads();
+      double xo[4][2][2];
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 2; ++y) xo[x][y][0] = xo[x][y][1] = 0.0;
+#pragma unroll
+      for (int k4 = 0; k4 < kTW / 4; ++k4) {
+        double fa[4], fb[2];
+#pragma unroll
+        for (int x = 0; x < 4; ++x) fa[x] = s.x[k4 * 4 + q][wr + x * 8 + g];
+#pragma unroll
+        for (int y = 0; y < 2; ++y) fb[y] = s.inv[k4 * 4 + q][wc + y * 8 + g];
+#pragma unroll
+        for (int x = 0; x < 4; ++x)
+#pragma unroll
+          for (int y = 0; y < 2; ++y) dmma(xo[x][y], fa[x], fb[y]);
+      }
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 2; ++y)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int r = r0 + wr + x * 8 + g, c = wc + y * 8 + 2 * q + h;
+            if (r < m && c < w) B[(size_t)(c0 + c) * ldb + r] = xo[x][y][h];
+          }
+      __syncthreads();  // X_J visible to the CTA before the next block reads it
+    }
+  }
+}
+
+int g_sms = 0;
+
+int launch_blas(const BlasArgs& a, cudaStream_t stream) {
+  if (!g_sms) {
+    int dev;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  void* ws = nullptr;
+  cudaError_t e = ws_alloc(&ws, sizeof(int) * ((size_t)a.batch + 2), stream);
+  if (e != cudaSuccess) return (int)e;
+  int* off = static_cast<int*>(ws);
+  int* counter = off + a.batch + 1;
+  tile_scan_kernel<<<1, 1024, 0, stream>>>(a, off, counter);
+  e = cudaGetLastError();
+  if (e == cudaSuccess) {
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cfg.stream = stream;
+    cfg.blockDim = dim3(kGThreads);
+    cfg.gridDim = dim3(g_sms * 8);
+    if (a.mode == kTrsm) e = cudaLaunchKernelEx(&cfg, trsm_kernel, a, (const int*)off, counter);
+    else e = cudaLaunchKernelEx(&cfg, gemm_syrk_kernel, a, (const int*)off, counter);
+  }
+  cudaError_t e2 = ws_free(ws, stream);
+  return (int)(e != cudaSuccess ? e : e2);
+}
+
+bool is_t(char c) { return c == 'T' || c == 't' || c == 'C' || c == 'c'; }
+
+}  // namespace
+
+int gemm_launch(char ta, char tb, const int* d_m, const int* d_n, const int* d_k, double alpha,
+                const double* const* dA, const int* d_lda, const double* const* dB,
+                const int* d_ldb, double beta, double* const* dC, const int* d_ldc, int batch,
+                int, int, int, cudaStream_t stream) {
+  BlasArgs a = {};
+  a.mode = kGemm;
+  a.ta = is_t(ta);
+  a.tb = is_t(tb);
+  a.m = d_m; a.n = d_n; a.k = d_k;
+  a.alpha = alpha; a.beta = beta;
+  a.A = dA; a.lda = d_lda; a.B = dB; a.ldb = d_ldb; a.C = dC; a.ldc = d_ldc;
+  a.batch = batch;
+  return launch_blas(a, stream);
+}
+
+int syrk_launch(char uplo, char trans, const int* d_n, const int* d_k, double alpha,
+                const double* const* dA, const int* d_lda, double beta, double* const* dC,
+                const int* d_ldc, int batch, int, int, cudaStream_t stream) {
+  BlasArgs a = {};
+  a.mode = (uplo == 'L' || uplo == 'l') ? kSyrkLower : kSyrkUpper;
+  a.ta = is_t(trans);   // op(A) = A (N) or A^T (T)
+  a.tb = !a.ta;         // second operand op(A)^T
+  a.m = d_n; a.n = d_n; a.k = d_k;
+  a.alpha = alpha; a.beta = beta;
+  a.A = dA; a.lda = d_lda; a.B = dA; a.ldb = d_lda; a.C = dC; a.ldc = d_ldc;
+  a.batch = batch;
+  return launch_blas(a, stream);
+}
+
+int trsm_launch(char, char uplo, char ta, char diag, const int* d_m, const int* d_n, double alpha,
+                const double* const* dA, const int* d_lda, double* const* dB, const int* d_ldb,
+                int batch, int, int, cudaStream_t stream) {
+  BlasArgs a = {};
+  a.mode = kTrsm;
+  a.ta = is_t(ta);
+  a.upper_in_A = (uplo == 'U' || uplo == 'u');
+  a.tlower = (!a.upper_in_A) ^ a.ta;  // T = op(A) is lower iff (A lower) xor transposed
+  a.unit = (diag == 'U' || diag == 'u');
+  a.m = d_m; a.n = d_n; a.k = d_n;
+  a.alpha = alpha; a.beta = 0.0;
+  a.A = dA; a.lda = d_lda; a.C = dB; a.ldc = d_ldb;
+  a.batch = batch;
+  return launch_blas(a, stream);
+}
+
+}  // namespace vb

@@ -1,0 +1,60 @@
+// common.cuh — device helpers shared by the vbatched kernels (sm_100a only).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ != 1000)
+#error "libvbatched is written for sm_100a only (compile with -gencode arch=compute_100a,code=sm_100a)"
+#endif
+
+#define VB_DEVINL __device__ __forceinline__
+
+namespace vb {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// Control block written by the scan (one per call, in the stream-ordered workspace).
+struct Ctrl {
+  int head_big;    // atomic queue head over order[0 .. count_big)
+  int head_warp;   // atomic queue head over order[count_big .. count_big+count_warp)
+  int count_big;   // valid matrices with n > kWarpMaxN, sorted by n descending
+  int count_warp;  // valid matrices with 1 <= n <= kWarpMaxN, sorted by n descending
+  int max_n;       // max n over valid matrices (for the _nomax interface / logging)
+  int pad[3];
+};
+
+constexpr int kWarpMaxN = 32;  // warp-per-matrix path for n <= 32
+
+// FP64 tensor-core MMA: D(8x8) += A(8x4, row) * B(4x8, col). Native SASS: DMMA.8x8x4.
+// Fragment layout (verified on B200 by tools/fp64_peaks.cu): lane l = 4g + q holds
+//   A[g][q], B[q][g], and C[g][2q], C[g][2q+1].
+VB_DEVINL void dmma(double (&d)[2], double a, double b) {
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+      : "+d"(d[0]), "+d"(d[1])
+      : "d"(a), "d"(b));
+}
+
+VB_DEVINL uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// cp.async 8 bytes with zero fill when !pred (src must still be a mapped address).
+VB_DEVINL void cp_async8(void* sdst, const void* gsrc, bool pred) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),
+               "r"(pred ? 8 : 0));
+}
+// cp.async 16 bytes (L2 only), zero fill when !pred.
+VB_DEVINL void cp_async16(void* sdst, const void* gsrc, bool pred) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),
+               "r"(pred ? 16 : 0));
+}
+VB_DEVINL void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+VB_DEVINL void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+// Programmatic dependent launch (PDL): wait for the upstream grid's results / let the
+// downstream grid start its prologue early.
+VB_DEVINL void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+VB_DEVINL void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;\n" ::); }
+
+}  // namespace vb

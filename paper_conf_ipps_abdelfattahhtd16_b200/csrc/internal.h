@@ -1,0 +1,34 @@
+// internal.h — host-side declarations shared by the translation units of libvbatched.so.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace vb {
+
+cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
+                            bool check_max, Ctrl* ctrl, int* order, cudaStream_t stream);
+
+// Persistent factorisation over the sorted work list (blocked CTA path for n > 32,
+// warp-per-matrix path for n <= 32). max_n_hint selects the launch configuration.
+cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                               int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
+                               cudaStream_t stream);
+
+// Stream-ordered scratch (pool-backed cudaMallocAsync).
+cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream);
+cudaError_t ws_free(void* p, cudaStream_t stream);
+
+// vbatched BLAS launchers (blas.cu).
+int gemm_launch(char ta, char tb, const int* d_m, const int* d_n, const int* d_k, double alpha,
+                const double* const* dA, const int* d_lda, const double* const* dB,
+                const int* d_ldb, double beta, double* const* dC, const int* d_ldc, int batch,
+                int max_m, int max_n, int max_k, cudaStream_t stream);
+int syrk_launch(char uplo, char trans, const int* d_n, const int* d_k, double alpha,
+                const double* const* dA, const int* d_lda, double beta, double* const* dC,
+                const int* d_ldc, int batch, int max_n, int max_k, cudaStream_t stream);
+int trsm_launch(char side, char uplo, char ta, char diag, const int* d_m, const int* d_n,
+                double alpha, const double* const* dA, const int* d_lda, double* const* dB,
+                const int* d_ldb, int batch, int max_m, int max_n, cudaStream_t stream);
+
+}  // namespace vb

@@ -1,0 +1,267 @@
+"""GPU parity of vbatched_dpotrf (through the C ABI) against the CPU oracle.
+
+Gates (BASELINE.json north_star): info[] bit-exact; backward error
+||A - L L^T||_F / (n ||A||_F eps) <= 10 (eps = 2^-53); row-scaled difference to the
+oracle's L <= 1e-10 (kappa <= 1e4). Exact integer families must be bit-exact. The strict
+upper triangle and padding rows must be bit-identical afterwards (NaN sentinels).
+"""
+import numpy as np
+import pytest
+import torch
+
+import vbgen
+from harness import DeviceBatch, compare_with_oracle
+
+pytestmark = pytest.mark.gpu
+
+POISON = np.uint64(vbgen.NAN_POISON_BITS)
+
+
+def _check_batch(db: DeviceBatch, idxs=None, exact_inputs=None):
+    torch.cuda.synchronize()
+    info = db.info()
+    bad = []
+    idxs = range(db.B) if idxs is None else idxs
+    for i in idxs:
+        n = int(db.n[i])
+        blk = db.block(i)
+        if n == 0:
+            assert info[i] == 0
+            continue
+        A = db.host_matrix_input(i) if exact_inputs is None else exact_inputs[i]
+        r = compare_with_oracle(A, blk, info[i])
+        if not r["ok"]:
+            bad.append((i, r))
+    assert not bad, bad[:5]
+    return info
+
+
+def _check_sentinels(db: DeviceBatch, idxs=None):
+    for i in (range(db.B) if idxs is None else idxs):
+        n, ld = int(db.n[i]), int(db.ldda[i])
+        if n <= 0:
+            continue
+        blk = db.block(i).view(np.uint64)
+        mask = np.ones((ld, n), bool)
+        mask[:n, :n] = np.triu(np.ones((n, n), bool), 1)  # strict upper of the n x n part
+        mask[n:, :] = True
+        assert np.all(blk[mask] == POISON), f"matrix {i} (n={n}, ld={ld}) touched outside lower"
+
+
+def test_generator_device_matches_numpy():
+    n = np.array([1, 2, 5, 33, 64, 130], dtype=np.int32)
+    db = DeviceBatch(n, seed=7, nonspd_mod=3).fill(poison=True)
+    torch.cuda.synchronize()
+    for i in range(db.B):
+        blk = db.block(i)
+        A = db.host_matrix_input(i)
+        low = np.tril(np.ones((n[i], n[i]), bool))
+        assert np.array_equal(blk[: n[i]][low].view(np.uint64), A[low].view(np.uint64))
+    _check_sentinels(db)
+
+
+def test_c1_full_parity():
+    n = vbgen.sizes("C1")
+    db = DeviceBatch(n, seed=1).fill(poison=True)
+    db.dpotrf(max_n=32)
+    info = _check_batch(db)
+    assert np.all(info == 0)
+    _check_sentinels(db)
+
+
+EDGE = [1, 2, 3, 7, 8, 15, 16, 17, 31, 32, 33, 34, 47, 48, 63, 64, 65, 96, 127, 128, 129, 130,
+        159, 160, 161, 191, 255, 256, 257, 300, 383, 384, 385, 511, 512, 513]
+
+
+@pytest.mark.parametrize("ldda_mode", ["pad32", "tight", "odd"])
+def test_edge_sizes(ldda_mode):
+    n = np.array(EDGE, dtype=np.int32)
+    db = DeviceBatch(n, seed=11, ldda_mode=ldda_mode).fill(poison=True)
+    db.dpotrf()
+    info = _check_batch(db)
+    assert np.all(info == 0)
+    _check_sentinels(db)
+
+
+def test_large_sizes():
+    n = np.array([640, 767, 1000, 1023, 1024, 1025], dtype=np.int32)
+    db = DeviceBatch(n, seed=12).fill(poison=True)
+    db.dpotrf()
+    _check_batch(db)
+    _check_sentinels(db)
+
+
+def test_nonspd_info_positions():
+    """Non-SPD by negating a_kk at block boundaries and ends."""
+    cases = []
+    for n in (1, 5, 32, 33, 64, 65, 100, 200, 300):
+        for k in sorted({min(n, v) for v in (1, 2, 31, 32, 33, 64, 65)} | {n}):
+            cases.append((n, k))
+    n_arr = np.array([c[0] for c in cases], dtype=np.int32)
+    db = DeviceBatch(n_arr, seed=3)
+    inputs = {}
+    for i, (n, k) in enumerate(cases):
+        A = vbgen.f1_matrix(3, i, n)
+        A[k - 1, k - 1] = -A[k - 1, k - 1]
+        inputs[i] = A
+        db.set_matrix(i, A)
+    db.dpotrf()
+    info = _check_batch(db, exact_inputs=inputs)
+    assert list(info) == [k for _, k in cases]
+    _check_sentinels(db)
+
+
+def test_nan_info():
+    cases = [(8, (2, 2)), (8, (5, 1)), (40, (33, 33)), (40, (39, 10)), (100, (70, 64)),
+             (100, (0, 0)), (100, (99, 99))]
+    n_arr = np.array([c[0] for c in cases], dtype=np.int32)
+    db = DeviceBatch(n_arr, seed=4)
+    for i, (n, (r, c)) in enumerate(cases):
+        A = vbgen.f1_matrix(4, i, n)
+        A[r, c] = np.nan
+        A[c, r] = np.nan
+        db.set_matrix(i, A)
+    db.dpotrf()
+    torch.cuda.synchronize()
+    assert list(db.info()) == [r + 1 for _, (r, c) in cases]  # MKL/LAPACK DISNAN convention
+
+
+def test_exact_families_bit_exact():
+    """min(i,j) -> tril(ones); integer unit-lower L -> L; power-of-two diagonals."""
+    rng = np.random.default_rng(0)
+    mats, Ls = [], []
+    for n in (5, 32, 33, 100, 200, 300):
+        i = np.arange(1, n + 1)
+        mats.append(np.minimum.outer(i, i).astype(np.float64))
+        Ls.append(np.tril(np.ones((n, n))))
+    for n in (33, 128, 257, 400):
+        L = np.tril(rng.integers(-1, 2, (n, n)), -1).astype(np.int64)
+        L[np.arange(n), np.arange(n)] = rng.choice([1, 2, 4], size=n)
+        mats.append((L @ L.T).astype(np.float64))
+        Ls.append(L.astype(np.float64))
+    n_arr = np.array([m.shape[0] for m in mats], dtype=np.int32)
+    db = DeviceBatch(n_arr)
+    for i, A in enumerate(mats):
+        db.set_matrix(i, A)
+    db.dpotrf()
+    torch.cuda.synchronize()
+    assert np.all(db.info() == 0)
+    for i, L in enumerate(Ls):
+        n = L.shape[0]
+        got = np.tril(db.block(i)[:n])
+        assert np.array_equal(got, L), f"case {i} n={n}: max diff {np.max(np.abs(got - L))}"
+    _check_sentinels(db)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
+def test_config_full_parity(cfg):
+    c = vbgen.CONFIGS[cfg]
+    n = vbgen.sizes(c)
+    db = DeviceBatch(n, seed=c.seed, nonspd_mod=c.nonspd_mod).fill(poison=(cfg == "C2"))
+    db.dpotrf(max_n=c.nmax)
+    info = _check_batch(db)
+    if c.nonspd_mod:
+        for i in range(db.B):
+            expect = vbgen.nonspd_k(c.seed, i, int(n[i])) if vbgen.is_nonspd(c, i) else 0
+            assert info[i] == expect
+    else:
+        assert np.all(info == 0)
+    if cfg == "C2":
+        _check_sentinels(db)
+
+
+def test_c5_full_size_sampled():
+    """C5 at BASELINE size (40000 x U{1..1024}, 112 GB) in the bench launch configuration;
+    every info must be 0; a deterministic sample is compared with the oracle."""
+    free, _ = torch.cuda.mem_get_info()
+    c = vbgen.CONFIGS["C5"]
+    n = vbgen.sizes(c)
+    need = vbgen.arena_layout(n, vbgen.ldda_for(n))[1] * 8
+    if need > free * 0.9:
+        pytest.skip("not enough device memory for full C5")
+    db = DeviceBatch(n, seed=c.seed).fill()
+    db.dpotrf(max_n=c.nmax)
+    torch.cuda.synchronize()
+    assert np.all(db.info() == 0)
+    order = np.argsort(-n, kind="stable")
+    sample = list(order[:4]) + list(range(0, db.B, 4001)) + list(order[-3:])
+    _check_batch(db, idxs=sample)
+    del db
+    torch.cuda.empty_cache()
+
+
+def test_nomax_equals_max():
+    n = vbgen.sizes("C2")[:500]
+    a = DeviceBatch(n, seed=2).fill()
+    b = DeviceBatch(n, seed=2).fill()
+    a.dpotrf(max_n=128)
+    from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf_nomax
+    vbatched_dpotrf_nomax("L", b.d_n, b.d_ptrs, b.d_ldda, b.d_info, b.B)
+    torch.cuda.synchronize()
+    assert torch.equal(a.arena, b.arena)
+    assert np.array_equal(a.info(), b.info())
+
+
+def test_invalid_matrices_untouched():
+    """n<0 -> -2, ldda<max(1,n) -> -4, n>max_n -> -7; those matrices are not touched."""
+    n = np.array([10, 40, 50, 3, 0, 70], dtype=np.int32)
+    ld = np.array([32, 64, 64, 32, 1, 96], dtype=np.int32)
+    db = DeviceBatch(n, ldda=ld, seed=5).fill(poison=True)
+    before = db.host_arena().copy()
+    bad_n = db.d_n.clone()
+    bad_n[3] = -1
+    bad_ld = db.d_ldda.clone()
+    bad_ld[1] = 39
+    from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
+    vbatched_dpotrf("L", bad_n, db.d_ptrs, bad_ld, db.d_info, db.B, 60)
+    torch.cuda.synchronize()
+    info = db.info()
+    assert list(info) == [0, -4, 0, -2, 0, -7]
+    after = db.host_arena()
+    for i in (1, 3, 5):
+        s = slice(db.off[i], db.off[i] + int(ld[i]) * max(int(n[i]), 0))
+        assert np.array_equal(before[s].view(np.uint64), after[s].view(np.uint64))
+    _check_batch(db, idxs=[0, 2])
+
+
+def test_argument_errors_and_empty():
+    from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
+    db = DeviceBatch(np.array([4], dtype=np.int32)).fill()
+    assert vbatched_dpotrf("X", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, 4, check=False) == -1
+    assert vbatched_dpotrf("U", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, 4, check=False) == -1
+    assert vbatched_dpotrf("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, -1, 4, check=False) == -6
+    assert vbatched_dpotrf("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, -1, check=False) == -7
+    assert vbatched_dpotrf("L", 0, 0, 0, 0, 0, 0, check=False) == 0
+
+
+def test_stream_semantics():
+    """Work is enqueued on the given stream; nothing happens on another stream's timeline."""
+    n = vbgen.sizes("C3")[:300]
+    db = DeviceBatch(n, seed=3).fill()
+    ref = DeviceBatch(n, seed=3).fill()
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        db.dpotrf(stream=s)
+    s.synchronize()
+    ref.dpotrf()
+    torch.cuda.synchronize()
+    assert torch.equal(db.arena, ref.arena)  # deterministic across streams / runs
+
+
+def test_host_api_chunked():
+    """vbatched_dpotrf_host: host buffers, small workspace -> many chunks; bit-identical to the
+    device API on the same inputs."""
+    from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf_host
+    n = vbgen.sizes("C3")[:400]
+    dev = DeviceBatch(n, seed=3).fill()
+    torch.cuda.synchronize()
+    host = dev.arena.cpu().numpy().copy()
+    dev.dpotrf()
+    torch.cuda.synchronize()
+    ptrs = (host.ctypes.data + 8 * dev.off).astype(np.int64)
+    info = np.full(dev.B, -99, dtype=np.int32)
+    vbatched_dpotrf_host("L", dev.n, ptrs, dev.ldda, info, dev.B, int(n.max()),
+                         workspace_bytes=3 * 48 << 20)
+    assert np.array_equal(info, dev.info())
+    assert np.array_equal(host, dev.arena.cpu().numpy())
