@@ -68,6 +68,26 @@ int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const in
 int vbatched_dpotrf_nomax(char uplo, const int* d_n, double* const* dA_array,
                           const int* d_ldda, int* d_info, int batchCount, vb_stream_t stream);
 
+/* Two-phase form of vbatched_dpotrf with caller-owned workspace (same arguments, same
+ * results; vbatched_dpotrf == scan + factor on an internal workspace):
+ *   vbatched_dpotrf_workspace_size(batchCount) -> bytes of device workspace needed;
+ *   vbatched_dpotrf_scan:   step a1 — validate n/ldda (writes info -2/-4/-7/0), compute the
+ *                           device max, counting-sort the valid matrices by n descending
+ *                           into the workspace;
+ *   vbatched_dpotrf_factor: steps a2-a7 — the persistent factorisation kernel draining the
+ *                           sorted work list written by the preceding scan on the same
+ *                           workspace (must follow it in stream order, once).
+ * d_workspace: device memory of at least vbatched_dpotrf_workspace_size bytes, 16-byte
+ * aligned, not used concurrently by another call. Return codes are minus the argument
+ * position in each function's own list (scan: uplo -1, batchCount -5, max_n -6, NULL
+ * workspace -7; factor: uplo -1, batchCount -6, max_n -7, NULL workspace -8). */
+size_t vbatched_dpotrf_workspace_size(int batchCount);
+int vbatched_dpotrf_scan(char uplo, const int* d_n, const int* d_ldda, int* d_info,
+                         int batchCount, int max_n, void* d_workspace, vb_stream_t stream);
+int vbatched_dpotrf_factor(char uplo, const int* d_n, double* const* dA_array,
+                           const int* d_ldda, int* d_info, int batchCount, int max_n,
+                           void* d_workspace, vb_stream_t stream);
+
 /* ---------------------------------------------------------------------------------------
  * vbatched_dpotrf_host — end-to-end variant on HOST memory (blocking).
  * Same problem and semantics as vbatched_dpotrf, but h_n, hA_array (host pointers to host
@@ -91,7 +111,7 @@ int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA_array, con
  *
  * vbatched_dgemm: C_i = alpha op(A_i) op(B_i) + beta C_i, C_i m_i x n_i, op(A_i) m_i x k_i.
  *   transA, transB in {'N','T'} (args 1,2). max_m/max_n/max_k >= every m_i/n_i/k_i
- *   (args 16-18; -p if < 0). beta == 0 does not read C. (DMMA tensor-core kernel.)
+ *   (args 15-17; -p if < 0; batchCount is arg 14). beta == 0 does not read C. (DMMA kernel.)
  */
 int vbatched_dgemm(char transA, char transB, const int* d_m, const int* d_n, const int* d_k,
                    double alpha, const double* const* dA_array, const int* d_ldda,

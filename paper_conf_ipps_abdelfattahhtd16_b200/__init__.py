@@ -16,7 +16,8 @@ import ctypes
 import os
 
 __all__ = [
-    "vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host", "vbatched_dgemm",
+    "vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
+    "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
     "vbatched_host_alloc", "vbatched_host_free", "lib", "LIB_PATH", "VBatchedError",
 ]
@@ -46,6 +47,10 @@ def lib() -> ctypes.CDLL:
         L = ctypes.CDLL(LIB_PATH)
         L.vbatched_dpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
         L.vbatched_dpotrf_nomax.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _vp]
+        L.vbatched_dpotrf_workspace_size.argtypes = [_i]
+        L.vbatched_dpotrf_workspace_size.restype = ctypes.c_size_t
+        L.vbatched_dpotrf_scan.argtypes = [_c, _vp, _vp, _vp, _i, _i, _vp, _vp]
+        L.vbatched_dpotrf_factor.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp, _vp]
         L.vbatched_dpotrf_host.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, ctypes.c_size_t, _vp]
         L.vbatched_dgemm.argtypes = [_c, _c, _vp, _vp, _vp, _d, _vp, _vp, _vp, _vp, _d, _vp, _vp,
                                      _i, _i, _i, _i, _vp]
@@ -58,6 +63,7 @@ def lib() -> ctypes.CDLL:
         L.vbatched_host_alloc.restype = _vp
         L.vbatched_host_free.argtypes = [_vp]
         for name in ("vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
+                     "vbatched_dpotrf_scan", "vbatched_dpotrf_factor",
                      "vbatched_dgemm", "vbatched_dsyrk", "vbatched_dtrsm",
                      "vbatched_partition_lpt", "vbatched_host_free"):
             getattr(L, name).restype = _i
@@ -107,6 +113,25 @@ def vbatched_dpotrf_nomax(uplo, n, dA_array, ldda, info, batchCount, stream=None
     rc = lib().vbatched_dpotrf_nomax(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
                                      int(batchCount), _stream(stream))
     return _check(rc, "vbatched_dpotrf_nomax") if check else rc
+
+
+def vbatched_dpotrf_workspace_size(batchCount) -> int:
+    return int(lib().vbatched_dpotrf_workspace_size(int(batchCount)))
+
+
+def vbatched_dpotrf_scan(uplo, n, ldda, info, batchCount, max_n, d_workspace, stream=None,
+                         check=True):
+    rc = lib().vbatched_dpotrf_scan(_ch(uplo), _ptr(n), _ptr(ldda), _ptr(info), int(batchCount),
+                                    int(max_n), _ptr(d_workspace), _stream(stream))
+    return _check(rc, "vbatched_dpotrf_scan") if check else rc
+
+
+def vbatched_dpotrf_factor(uplo, n, dA_array, ldda, info, batchCount, max_n, d_workspace,
+                           stream=None, check=True):
+    rc = lib().vbatched_dpotrf_factor(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
+                                      int(batchCount), int(max_n), _ptr(d_workspace),
+                                      _stream(stream))
+    return _check(rc, "vbatched_dpotrf_factor") if check else rc
 
 
 def vbatched_dpotrf_host(uplo, h_n, hA_array, h_ldda, h_info, batchCount, max_n,

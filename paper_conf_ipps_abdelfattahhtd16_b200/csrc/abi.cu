@@ -72,6 +72,35 @@ int vbatched_dpotrf_nomax(char uplo, const int* d_n, double* const* dA_array, co
                     (cudaStream_t)stream);
 }
 
+size_t vbatched_dpotrf_workspace_size(int batchCount) {
+  return sizeof(Ctrl) + sizeof(int) * (size_t)(batchCount > 0 ? batchCount : 0);
+}
+
+int vbatched_dpotrf_scan(char uplo, const int* d_n, const int* d_ldda, int* d_info, int batchCount,
+                         int max_n, void* d_workspace, vb_stream_t stream) {
+  if (uplo != 'L' && uplo != 'l') return -1;
+  if (batchCount < 0) return -5;
+  if (max_n < 0) return -6;
+  if (batchCount == 0) return 0;
+  if (!d_workspace) return -7;
+  Ctrl* ctrl = static_cast<Ctrl*>(d_workspace);
+  return (int)launch_scan_bin(d_n, d_ldda, d_info, batchCount, max_n, true, ctrl,
+                              reinterpret_cast<int*>(ctrl + 1), (cudaStream_t)stream);
+}
+
+int vbatched_dpotrf_factor(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
+                           int* d_info, int batchCount, int max_n, void* d_workspace,
+                           vb_stream_t stream) {
+  if (uplo != 'L' && uplo != 'l') return -1;
+  if (batchCount < 0) return -6;
+  if (max_n < 0) return -7;
+  if (batchCount == 0 || max_n == 0) return 0;
+  if (!d_workspace) return -8;
+  Ctrl* ctrl = static_cast<Ctrl*>(d_workspace);
+  return (int)launch_potrf_paths(d_n, dA_array, d_ldda, d_info, batchCount, max_n, ctrl,
+                                 reinterpret_cast<int*>(ctrl + 1), (cudaStream_t)stream);
+}
+
 int vbatched_dgemm(char transA, char transB, const int* d_m, const int* d_n, const int* d_k,
                    double alpha, const double* const* dA_array, const int* d_ldda,
                    const double* const* dB_array, const int* d_lddb, double beta,
