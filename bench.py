@@ -242,7 +242,7 @@ def our_arm(args, cfg, rank, world, local_rank):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
     max_n = int(n_all.max())
-    launches_per_step = 2  # scan_bin_kernel + potrf_persistent_kernel
+    launches_per_step = 3 if max_n > 32 else 2  # scan_bin + potrf_blocked + potrf_warp
 
     def prepare():
         db.fill()
@@ -308,7 +308,7 @@ def our_arm(args, cfg, rank, world, local_rank):
     roof["traffic"] = tr.get("bytes_per_launch") if tr else None
     if tr:
         roof["traffic_source"] = tr.get("source")
-    roof["kernel"] = "potrf_persistent_kernel<true>" if max_n > 32 else "potrf_persistent_kernel<false>"
+    roof["kernel"] = "potrf_blocked_kernel + potrf_warp_kernel" if max_n > 32 else "potrf_warp_kernel"
     roof["kernel_ms"] = sum(kern_ms) / args.steps
     roof["scan_ms"] = (sum(step_ms) - sum(kern_ms)) / args.steps
 
