@@ -149,6 +149,10 @@ int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owne
 /* Library version string and the tuning constants compiled in (for logs). */
 const char* vbatched_version(void);
 
+/* Number of kernel launches one vbatched_dpotrf call with this max_n enqueues (the scan plus
+ * one persistent kernel per non-empty size range). For benchmarks' launch accounting. */
+int vbatched_dpotrf_kernel_launches(int max_n);
+
 /* Pinned host memory helpers (cudaHostAlloc / cudaFreeHost) for the _host entry point. */
 void* vbatched_host_alloc(size_t bytes);
 int vbatched_host_free(void* p);

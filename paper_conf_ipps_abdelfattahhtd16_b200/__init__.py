@@ -19,11 +19,11 @@ __all__ = [
     "vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
     "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
-    "vbatched_host_alloc", "vbatched_host_free", "lib", "LIB_PATH", "VBatchedError",
+    "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "lib", "LIB_PATH", "VBatchedError",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libvbatched.so")
+LIB_PATH = os.environ.get("VBATCHED_LIB", os.path.join(_HERE, "libvbatched.so"))
 
 _vp = ctypes.c_void_p
 _i = ctypes.c_int
@@ -59,6 +59,8 @@ def lib() -> ctypes.CDLL:
                                      _vp]
         L.vbatched_partition_lpt.argtypes = [_vp, _i, _i, _vp]
         L.vbatched_version.restype = ctypes.c_char_p
+        L.vbatched_dpotrf_kernel_launches.argtypes = [_i]
+        L.vbatched_dpotrf_kernel_launches.restype = _i
         L.vbatched_host_alloc.argtypes = [ctypes.c_size_t]
         L.vbatched_host_alloc.restype = _vp
         L.vbatched_host_free.argtypes = [_vp]
@@ -176,6 +178,10 @@ def vbatched_partition_lpt(h_n, ngpu: int):
     _check(lib().vbatched_partition_lpt(_ptr(h_n), len(h_n), int(ngpu), _ptr(owner)),
            "vbatched_partition_lpt")
     return owner
+
+
+def vbatched_dpotrf_kernel_launches(max_n: int) -> int:
+    return int(lib().vbatched_dpotrf_kernel_launches(int(max_n)))
 
 
 def vbatched_version() -> str:

@@ -167,9 +167,15 @@ int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owne
 }
 
 const char* vbatched_version(void) {
-  return "libvbatched 0.1 (sm_100a; blocked NB=32 MB=128 KC=16 stages=3; warp path n<=32; "
-         "DMMA m8n8k4 f64)";
+  static char buf[256];
+  snprintf(buf, sizeof buf,
+           "libvbatched 0.2 (sm_100a; DMMA m8n8k4 f64; blocked NB=64 for n>%d, NB=32 for "
+           "32<n<=%d, MB=128; warp path n<=32)",
+           potrf_t64(), potrf_t64());
+  return buf;
 }
+
+int vbatched_dpotrf_kernel_launches(int max_n) { return max_n > 0 ? potrf_num_launches(max_n) : 0; }
 
 void* vbatched_host_alloc(size_t bytes) {
   void* p = nullptr;

@@ -14,13 +14,17 @@ namespace vb {
 constexpr unsigned kFull = 0xffffffffu;
 
 // Control block written by the scan (one per call, in the stream-ordered workspace).
+// The sorted work list order[] holds the valid matrices by n descending, split in three
+// contiguous ranges, one per factorisation kernel:
+//   range 0: n > t64        (blocked kernel, panel width 64)
+//   range 1: 32 < n <= t64  (blocked kernel, panel width 32)
+//   range 2: 1 <= n <= 32   (warp-per-matrix kernel)
 struct Ctrl {
-  int head_big;    // atomic queue head over order[0 .. count_big)
-  int head_warp;   // atomic queue head over order[count_big .. count_big+count_warp)
-  int count_big;   // valid matrices with n > kWarpMaxN, sorted by n descending
-  int count_warp;  // valid matrices with 1 <= n <= kWarpMaxN, sorted by n descending
-  int max_n;       // max n over valid matrices (for the _nomax interface / logging)
-  int pad[3];
+  int head[3];   // atomic queue heads (per range)
+  int count[3];  // matrices per range
+  int start[3];  // first position of each range in order[]
+  int max_n;     // max n over valid matrices (for the _nomax interface / logging)
+  int pad[2];
 };
 
 constexpr int kWarpMaxN = 32;  // warp-per-matrix path for n <= 32

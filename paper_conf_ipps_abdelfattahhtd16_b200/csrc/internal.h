@@ -6,6 +6,9 @@
 
 namespace vb {
 
+// Size threshold above which matrices take the NB=64 blocked kernel (env VB_T64 overrides).
+int potrf_t64();
+
 cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
                             bool check_max, Ctrl* ctrl, int* order, cudaStream_t stream);
 
@@ -14,6 +17,8 @@ cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int 
 cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
                                cudaStream_t stream);
+
+int potrf_num_launches(int max_n_hint);
 
 // Stream-ordered scratch (pool-backed cudaMallocAsync).
 cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream);

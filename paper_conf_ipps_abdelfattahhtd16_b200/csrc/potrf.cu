@@ -1,62 +1,74 @@
 // potrf.cu — the factorisation kernels of vbatched_dpotrf (steps a2-a7 of SURVEY.md §8(a)).
 //
-// Two persistent kernels drain the work list written by scan_bin (matrices sorted by n
-// descending = flops descending, i.e. longest-processing-time first):
+// Three persistent kernels drain the three ranges of the work list written by scan_bin
+// (matrices sorted by n descending = flops descending: longest-processing-time first):
 //
-//  * potrf_blocked_kernel, n > 32: one CTA (8 warps) per matrix, the left-looking blocked
-//    Cholesky of PAPER.md Algorithm 1 with panel width NB = 32:
+//  * potrf_blocked_kernel<Cfg64>, n > t64, and potrf_blocked_kernel<Cfg32>, 32 < n <= t64:
+//    one CTA (8 warps) per matrix, the left-looking blocked Cholesky of PAPER.md Algorithm 1
+//     with panel width NB = 64 or 32:
 //      for each panel j0 (columns j0..j0+NB-1), for each block of MB = 128 rows r0 >= j0:
 //        panel update    C = A[r0:, j0:j0+NB] - L[r0:, 0:j0] L[j0:j0+NB, 0:j0]^T
 //                        ("customized syrk" with B a part of A, Fig. 2) on
-//                        the FP64 tensor cores (DMMA), operands staged by a 3-stage cp.async
+//                        the FP64 tensor cores (DMMA m8n8k4), operands staged by a cp.async
 //                        pipeline (double buffering); the accumulators start
 //                        from A's panel values, loaded before the k loop;
-//        tile factorize  L11 = chol(C1): POTF2 by one warp on the 32x32 block in shared
-//                        memory (row-owner lanes, LDL^T-form right-looking update so that
-//                        sqrt and the column scaling are off the column-to-column chain);
-//        panel factorize C2 <- C2 L11^-T: TRTRI of L11 by recursive doubling on DMMA in
-//                        shared memory, then a DMMA GEMM — the trtri + gemm TRSM design of
-//                        PAPER.md:760-772.
-//    Every element of L is written once; earlier columns are re-read once per panel.
-//  * potrf_warp_kernel, n <= 32: one warp per matrix, whole matrix in shared memory
-//    (the fused on-chip POTF2 of PAPER.md:551-560; one HBM read, one HBM write). It is
-//    launched after the blocked kernel with programmatic dependent launch and starts on the
-//    SMs the blocked kernel's CTAs free once its work list is empty (the smallest matrices
-//    come last in LPT order anyway).
+//        tile factorize  L11 = chol(C1): POTF2 of 32-wide blocks by one warp, rows in
+//                        registers (LDL^T-form right-looking update so that sqrt and the
+//                        column scaling stay off the column-to-column chain); for NB = 64 the
+//                        64x64 block is done as POTF2(32) / TRSM / SYRK / POTF2(32);
+//        panel factorize C2 <- C2 L11^-T: TRTRI of L11 in shared memory (8x8 substitution +
+//                        recursive doubling on DMMA), then a DMMA GEMM — the trtri + gemm
+//                        TRSM design of PAPER.md:760-772.
+//    Every element of L is written once; earlier columns are re-read once per panel, so the
+//    HBM re-read traffic is ~ 8 n^3 / (6 NB) bytes per matrix: the wider panel is used
+//    where matrices are large enough to keep its longer diagonal chain amortised.
+//  * potrf_warp_kernel, n <= 32: one warp per matrix, whole matrix in registers
+//    (the fused on-chip POTF2 of PAPER.md:551-560; one HBM read, one HBM write).
+// The kernels are chained with programmatic dependent launch: each releases its dependent
+// grid as soon as it starts, so the next range's CTAs take the SMs the previous kernel's
+// CTAs free at its tail (the smaller matrices come later in LPT order anyway).
 // Failed matrices (pivot <= 0 or NaN) stop at the failing column and report the LAPACK info
 // (SURVEY.md §8(c) readings #2-#3); nothing of them is touched again (a7).
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "internal.h"
 
 namespace vb {
 
-constexpr int NB = 32;       // panel width (Algorithm 1's nb)
-constexpr int MB = 128;      // rows per GEMM/TRSM pass (8 warps x 16 rows)
-constexpr int KC = 16;       // k-chunk per pipeline stage
-constexpr int STAGES = 3;    // cp.async pipeline depth
-constexpr int kThreads = 256;
-constexpr int LDA_S = MB + 4;  // padded smem leading dims (conflict-free DMMA fragment loads)
-constexpr int LDB_S = NB + 4;
-constexpr int LDI = NB + 4;
-constexpr int LDS_S = 20;      // TRTRI scratch
+template <int NB_, int MB_, int WARPS_M_, int WARPS_N_, int KC_, int STAGES_, int MINB_>
+struct BlockedCfg {
+  static constexpr int NB = NB_, MB = MB_, WARPS_M = WARPS_M_, WARPS_N = WARPS_N_;
+  static constexpr int KC = KC_, STAGES = STAGES_, MINB = MINB_;
+  static constexpr int THREADS = 32 * WARPS_M * WARPS_N;
+  static constexpr int WM = MB / WARPS_M, WN = NB / WARPS_N;
+  static constexpr int MT = WM / 8, NT = WN / 8;
+  static constexpr int LDA = MB + 4;  // padded smem leading dims: conflict-free fragments
+  static constexpr int LDB = NB + 4;
+  static constexpr int LDI = NB + 4;
+};
+using Cfg32 = BlockedCfg<32, 128, 8, 1, 16, 3, 3>;
+using Cfg64 = BlockedCfg<64, 128, 4, 2, 16, 2, 2>;
 
-struct BigSmem {
+constexpr int LDS_T = 20;  // TRTRI32 scratch leading dim
+
+template <class C>
+struct BlockedSmem {
   union {
     struct {
-      double a[STAGES][KC][LDA_S];  // A chunk: [k][row]
-      double b[STAGES][KC][LDB_S];  // B chunk: [k][panel row]
+      double a[C::STAGES][C::KC][C::LDA];  // A chunk: [k][row]
+      double b[C::STAGES][C::KC][C::LDB];  // B chunk: [k][panel row]
     } pipe;
     struct {
-      double tile[NB][LDA_S];  // C tile: [col][row], aliases the pipeline after the k loop
-      double scratch[16 * LDS_S * 2];  // TRTRI scratch
+      double tile[C::NB][C::LDA];  // C tile: [col][row], aliases the pipeline after the k loop
+      double scratch[16 * LDS_T * 2];  // TRTRI32 scratch
+      double wbuf[64];
+      double sv[C::NB];
+      double tv[C::NB];
     } e;
   } u;
-  double inv[NB][LDI];      // inv[k][n] = (L11^-1)[n][k]  (DMMA B operand of the TRSM)
-  double wbuf[2 * NB];
-  double sv[NB];
-  double tv[NB];
+  double inv[C::NB][C::LDI];  // inv[k][n] = (L11^-1)[n][k]  (DMMA B operand of the TRSM)
   int item;
   int info;
 };
@@ -117,14 +129,16 @@ VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws, dou
 }
 
 // ---------------------------------------------------------------------------------------
-// Inverse of the 32x32 lower-triangular L (T[c*ldt+r] = L[r][c], tv[c] = 1/L[c][c]) by one
+// Inverse of a 32x32 lower-triangular L (T[c*ldt+r] = L[r][c], tv[c] = 1/L[c][c]) by one
 // warp: 8x8 diagonal blocks by substitution (lane = block column), then two levels of
 // recursive doubling inv([[A,0],[B,C]]) = [[inv A, 0], [-inv C B inv A, inv C]] on DMMA.
-// Output INV[k*ldi + n] = X[n][k], X = L^-1 (the TRSM's B operand layout).
+// Output INV[k*ldi + n] = X[n][k], X = L^-1 (the TRSM's B operand layout); the 32x32 block
+// of INV is fully written (zeros above the diagonal of X). S: 16 x LDS_T x 2 doubles with
+// leading dimension lds.
 VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, double* INV,
-                                 int ldi, double* S, int lane) {
+                                 int ldi, double* S, int lds, int lane) {
   const int g = lane >> 2, q = lane & 3;
-  for (int e = lane; e < NB * NB; e += 32) INV[(e >> 5) * ldi + (e & 31)] = 0.0;
+  for (int e = lane; e < 32 * 32; e += 32) INV[(e >> 5) * ldi + (e & 31)] = 0.0;
   __syncwarp();
   {  // level 0: column c of inv(D_b), D_b = L[8b:8b+8, 8b:8b+8]
     const int b = lane >> 3, c = lane & 7, o = 8 * b;
@@ -149,15 +163,15 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
       const int o = 16 * p;
 #pragma unroll
       for (int ks = 0; ks < 2; ++ks) {
-        const double a = T[(o + ks * 4 + q) * ldt + o + 8 + g];   // B[g][k]
-        const double bb = INV[(o + g) * ldi + o + ks * 4 + q];    // invA[k][g]
+        const double a = T[(o + ks * 4 + q) * ldt + o + 8 + g];  // B[g][k]
+        const double bb = INV[(o + g) * ldi + o + ks * 4 + q];   // invA[k][g]
         dmma(t[p], a, bb);
       }
     }
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
-      S[p * 8 * LDS_S + g * LDS_S + 2 * q] = t[p][0];
-      S[p * 8 * LDS_S + g * LDS_S + 2 * q + 1] = t[p][1];
+      S[(p * 8 + g) * lds + 2 * q] = t[p][0];
+      S[(p * 8 + g) * lds + 2 * q + 1] = t[p][1];
     }
     __syncwarp();
     double r[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
@@ -167,7 +181,7 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
 #pragma unroll
       for (int ks = 0; ks < 2; ++ks) {
         const double a = INV[(o + 8 + ks * 4 + q) * ldi + o + 8 + g];  // invC[g][k]
-        const double bb = S[p * 8 * LDS_S + (ks * 4 + q) * LDS_S + g];  // Tm[k][g]
+        const double bb = S[(p * 8 + ks * 4 + q) * lds + g];            // Tm[k][g]
         dmma(r[p], a, bb);
       }
     }
@@ -202,8 +216,8 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
     for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
       for (int nt = 0; nt < 2; ++nt) {
-        S[(mt * 8 + g) * LDS_S + nt * 8 + 2 * q] = t[mt][nt][0];
-        S[(mt * 8 + g) * LDS_S + nt * 8 + 2 * q + 1] = t[mt][nt][1];
+        S[(mt * 8 + g) * lds + nt * 8 + 2 * q] = t[mt][nt][0];
+        S[(mt * 8 + g) * lds + nt * 8 + 2 * q + 1] = t[mt][nt][1];
       }
     __syncwarp();
     double r[2][2][2];
@@ -217,7 +231,7 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
 #pragma unroll
       for (int mt = 0; mt < 2; ++mt) a[mt] = INV[(16 + ks * 4 + q) * ldi + 16 + mt * 8 + g];
 #pragma unroll
-      for (int nt = 0; nt < 2; ++nt) bb[nt] = S[(ks * 4 + q) * LDS_S + nt * 8 + g];
+      for (int nt = 0; nt < 2; ++nt) bb[nt] = S[(ks * 4 + q) * lds + nt * 8 + g];
 #pragma unroll
       for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
@@ -234,50 +248,261 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
   __syncwarp();
 }
 
+// One warp: POTF2 of the nb x nb (nb <= 32) lower block at T (T[c*ldt + r]) in registers,
+// written back to T and to global (Ag, lda) — lower part, on failure up to the failing
+// column (incl. the pivot). Returns info.
+VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, int lda,
+                            double* ws, double* sv, double* tv) {
+  double a[32];
+#pragma unroll
+  for (int c = 0; c < 32; ++c) a[c] = T[c * ldt + lane];
+  const int info = potf2_regs_warp<32>(a, nb, lane, ws, sv, tv);
+  const int ncol = info ? info : nb;
+#pragma unroll
+  for (int c = 0; c < 32; ++c)
+    if (c < ncol && lane >= c && lane < nb) {
+      T[c * ldt + lane] = a[c];
+      Ag[(size_t)c * lda + lane] = a[c];
+    }
+  __syncwarp();
+  return info;
+}
+
+// Diagonal block, NB = 32 (warp 0 only). Sets s.info; builds s.inv when rows follow below.
+// Out of line so that its register footprint does not spill into the caller's k-loop.
+__device__ __noinline__ void diag_block32(BlockedSmem<Cfg32>& s, int nb, int lane, double* Ad,
+                                          int ld, bool below) {
+  const int info = potf2_block32(&s.u.e.tile[0][0], Cfg32::LDA, nb, lane, Ad, ld, s.u.e.wbuf,
+                                 s.u.e.sv, s.u.e.tv);
+  if (!info && below)
+    trtri32_dmma_warp(&s.u.e.tile[0][0], Cfg32::LDA, s.u.e.tv, &s.inv[0][0], Cfg32::LDI,
+                      s.u.e.scratch, LDS_T, lane);
+  if (lane == 0) s.info = info;
+}
+
+// 32x32x32 DMMA products on a 4-warp group (wg = warp index 0..3): each warp owns a 16x16
+// quarter (2x2 tiles). acc[m][n] += sum_k fa(m,k) fb(k,n) over k = 0..31.
+template <class FA, class FB>
+VB_DEVINL void mm32_quarter(double (&acc)[2][2][2], int wg, int lane, FA fa, FB fb) {
+  const int g = lane >> 2, q = lane & 3;
+  const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
+#pragma unroll
+  for (int ks = 0; ks < 8; ++ks) {
+    double a[2], b[2];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt) a[mt] = fa(m0 + mt * 8 + g, ks * 4 + q);
+#pragma unroll
+    for (int nt = 0; nt < 2; ++nt) b[nt] = fb(ks * 4 + q, n0 + nt * 8 + g);
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt) dmma(acc[mt][nt], a[mt], b[nt]);
+  }
+}
+
+VB_DEVINL void bar_group(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// Diagonal block, NB = 64, by warps 0..3 (named barrier 1, 128 threads):
+//   L11 = potf2(C11); L21 = C21 inv(L11)^T; C22 -= L21 L21^T; L22 = potf2(C22).
+// For the TRSM of the rows below (two 32-column steps, 32x32 inverses only, as PAPER.md:
+// 762-766 prescribes) it leaves in s.inv: inv(L11) in [0:32][0:32], L21^T in [0:32][32:64]
+// (inv[k][32+n] = L21[n][k]) and inv(L22) in [32:64][32:64], all as B operands
+// (inv[k][n] = X[n][k]). T = the C tile (T[c*LDA + r]). Sets s.info (1-based, in-block).
+__device__ __noinline__ void diag_block64(BlockedSmem<Cfg64>& s, int nb, int wg, int lane,
+                                          double* Ad, int ld, bool below) {
+  constexpr int LDA = Cfg64::LDA, LDI = Cfg64::LDI;
+  double* T = &s.u.e.tile[0][0];
+  double* INV = &s.inv[0][0];
+  const int g = lane >> 2, q = lane & 3;
+  const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
+  const int nb1 = min(nb, 32), nb2 = nb - nb1;
+  // (1) L11 = potf2(C11) and inv(L11) (warp 0); TRTRI scratch in INV[32:48][0:20] (unused)
+  if (wg == 0) {
+    const int info = potf2_block32(T, LDA, nb1, lane, Ad, ld, s.u.e.wbuf, s.u.e.sv, s.u.e.tv);
+    if (!info && nb2 > 0) trtri32_dmma_warp(T, LDA, s.u.e.tv, INV, LDI, INV + 32 * LDI, LDI, lane);
+    if (lane == 0) s.info = info;
+  }
+  bar_group(1, 128);
+  if (s.info || nb2 == 0) return;
+  // (2) L21 = C21 inv(L11)^T  (C21 = T rows 32..63, cols 0..31); B[k][n] = X11[n][k] = INV[k][n]
+  {
+    double acc[2][2][2] = {};
+    mm32_quarter(acc, wg, lane, [&](int m, int k) { return T[k * LDA + 32 + m]; },
+                 [&](int k, int n) { return INV[k * LDI + n]; });
+    bar_group(1, 128);  // all reads of C21 done
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
+          T[c * LDA + r] = acc[mt][nt][h];
+          INV[c * LDI + r] = acc[mt][nt][h];  // L21^T: inv[k=c][32+n] with n = r-32
+          if (r < nb) Ad[(size_t)c * ld + r] = acc[mt][nt][h];
+        }
+  }
+  bar_group(1, 128);
+  // (3) C22 -= L21 L21^T (T rows/cols 32..63)
+  {
+    double acc[2][2][2];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          acc[mt][nt][h] = T[(32 + n0 + nt * 8 + 2 * q + h) * LDA + 32 + m0 + mt * 8 + g];
+    mm32_quarter(acc, wg, lane, [&](int m, int k) { return -T[k * LDA + 32 + m]; },
+                 [&](int k, int n) { return T[k * LDA + 32 + n]; });
+    bar_group(1, 128);
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          T[(32 + n0 + nt * 8 + 2 * q + h) * LDA + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
+  }
+  bar_group(1, 128);
+  // (4) L22 = potf2(C22) and inv(L22) (warp 0); TRTRI scratch in INV[32:48][0:20] (unused)
+  if (wg == 0) {
+    double* T22 = T + 32 * LDA + 32;
+    const int info = potf2_block32(T22, LDA, nb2, lane, Ad + (size_t)32 * ld + 32, ld,
+                                   s.u.e.wbuf, s.u.e.sv + 32, s.u.e.tv + 32);
+    if (!info && below)
+      trtri32_dmma_warp(T22, LDA, s.u.e.tv + 32, INV + 32 * LDI + 32, LDI, INV + 32 * LDI, LDI,
+                        lane);
+    if (lane == 0) s.info = info ? 32 + info : 0;
+  }
+  bar_group(1, 128);
+}
+
 // Stage k-chunk kc of the panel-update operands: A rows r0..r0+MB-1 and the panel rows
 // j0..j0+NB-1 (the "B" of Fig. 2), columns kc*KC..kc*KC+KC-1. Rows >= n are zero-filled.
-VB_DEVINL void load_stage(BigSmem& s, int st, int kc, const double* __restrict__ A, int n, int ld,
-                          int r0, int j0) {
+template <class C>
+VB_DEVINL void load_stage(BlockedSmem<C>& s, int st, int kc, const double* __restrict__ A, int n,
+                          int ld, int r0, int j0) {
   const int tid = threadIdx.x;
-  const int k0 = kc * KC;
+  const int k0 = kc * C::KC;
 #pragma unroll
-  for (int e = 0; e < (MB * KC) / kThreads; ++e) {
-    const int idx = tid + e * kThreads;
-    const int c = idx / MB, r = idx % MB;
+  for (int e = 0; e < (C::MB * C::KC) / C::THREADS; ++e) {
+    const int idx = tid + e * C::THREADS;
+    const int c = idx / C::MB, r = idx % C::MB;
     const int row = r0 + r;
     const bool p = row < n;
     cp_async8(&s.u.pipe.a[st][c][r], A + (p ? (size_t)(k0 + c) * ld + row : 0), p);
   }
 #pragma unroll
-  for (int e = 0; e < (NB * KC) / kThreads; ++e) {
-    const int idx = tid + e * kThreads;
-    const int c = idx / NB, r = idx % NB;
+  for (int e = 0; e < (C::NB * C::KC) / C::THREADS; ++e) {
+    const int idx = tid + e * C::THREADS;
+    const int c = idx / C::NB, r = idx % C::NB;
     const int row = j0 + r;
     const bool p = row < n;
     cp_async8(&s.u.pipe.b[st][c][r], A + (p ? (size_t)(k0 + c) * ld + row : 0), p);
   }
 }
 
-// Blocked left-looking Cholesky of one matrix by the whole CTA.
-VB_DEVINL void potrf_big_matrix(BigSmem& s, double* __restrict__ A, int n, int ld,
-                                int* info_out) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+// TRSM of the 128 x NB C tile by its warps (warp w owns rows 16w..16w+15), in place.
+// B operands from s.inv (see diag_block64 / trtri32_dmma_warp for the layout).
+template <class C>
+VB_DEVINL void trsm_rows16(BlockedSmem<C>& s, int warp, int lane, bool active) {
   const int g = lane >> 2, q = lane & 3;
-  for (int j0 = 0; j0 < n; j0 += NB) {
-    const int nb = min(NB, n - j0);
-    const int nk = j0 / KC;
-    for (int r0 = j0; r0 < n; r0 += MB) {
-      const bool first = (r0 == j0);
-      const bool warp_active = (r0 + warp * 16) < n;
-      // ---- accumulators start from A's panel values (lower triangle only)
-      double acc[2][4][2];
+  const int r = warp * 16;
+  if (!active) return;
+#pragma unroll
+  for (int half = 0; half < C::NB / 32; ++half) {
+    const int c0 = half * 32;
+    double x[2][4][2];
+    if (half == 0) {
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) x[mt][nt][0] = x[mt][nt][1] = 0.0;
+    } else {
+      // C2 -= X1 L21^T  (acc from the tile's C2, A = X1 (tile cols 0..31), B = inv[k][32+n])
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h)
+            x[mt][nt][h] = s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g];
+#pragma unroll
+      for (int k4 = 0; k4 < 8; ++k4) {
+        double fa[2], fb[4];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.u.e.tile[k4 * 4 + q][r + mt * 8 + g];
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) fb[nt] = s.inv[k4 * 4 + q][32 + nt * 8 + g];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+      }
 #pragma unroll
       for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
         for (int nt = 0; nt < 4; ++nt)
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
-            const int row = r0 + warp * 16 + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
+            s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g] = x[mt][nt][h];
+            x[mt][nt][h] = 0.0;
+          }
+      __syncwarp();
+    }
+    // X_half = C_half inv(L_half,half)^T
+#pragma unroll
+    for (int k4 = 0; k4 < 8; ++k4) {
+      double fa[2], fb[4];
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt) fa[mt] = s.u.e.tile[c0 + k4 * 4 + q][r + mt * 8 + g];
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) fb[nt] = s.inv[c0 + k4 * 4 + q][c0 + nt * 8 + g];
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g] = x[mt][nt][h];
+    __syncwarp();
+  }
+}
+
+// Blocked left-looking Cholesky of one matrix by the whole CTA.
+template <class C>
+VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, int n, int ld,
+                                    int* info_out) {
+  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES;
+  constexpr int MT = C::MT, NT = C::NT;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  const int wrow = (warp % C::WARPS_M) * C::WM;  // warp's first row within the block
+  const int wcol = (warp / C::WARPS_M) * C::WN;  // warp's first panel column
+  for (int j0 = 0; j0 < n; j0 += NB) {
+    const int nb = min(NB, n - j0);
+    const int nk = j0 / KC;
+    for (int r0 = j0; r0 < n; r0 += MB) {
+      const bool first = (r0 == j0);
+      const bool warp_active = (r0 + wrow) < n;
+      // ---- accumulators start from A's panel values (lower triangle only)
+      double acc[MT][NT][2];
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int row = r0 + wrow + mt * 8 + g, col = j0 + wcol + nt * 8 + 2 * q + h;
             const bool v = row < n && col < j0 + nb && row >= col;
             acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
           }
@@ -285,30 +510,30 @@ VB_DEVINL void potrf_big_matrix(BigSmem& s, double* __restrict__ A, int n, int l
       if (nk > 0) {
 #pragma unroll
         for (int st = 0; st < STAGES - 1; ++st) {
-          if (st < nk) load_stage(s, st, st, A, n, ld, r0, j0);
+          if (st < nk) load_stage<C>(s, st, st, A, n, ld, r0, j0);
           cp_async_commit();
         }
         for (int kc = 0; kc < nk; ++kc) {
           cp_async_wait<STAGES - 2>();
           __syncthreads();
           const int pf = kc + STAGES - 1;
-          if (pf < nk) load_stage(s, pf % STAGES, pf, A, n, ld, r0, j0);
+          if (pf < nk) load_stage<C>(s, pf % STAGES, pf, A, n, ld, r0, j0);
           cp_async_commit();
           const int st = kc % STAGES;
           if (warp_active) {
 #pragma unroll
             for (int kk = 0; kk < KC / 4; ++kk) {
-              const double* sa = &s.u.pipe.a[st][kk * 4 + q][warp * 16 + g];
-              const double a0 = -sa[0], a1 = -sa[8];
-              const double* sb = &s.u.pipe.b[st][kk * 4 + q][g];
-              double b[4];
+              double fa[MT], fb[NT];
 #pragma unroll
-              for (int nt = 0; nt < 4; ++nt) b[nt] = sb[nt * 8];
+              for (int mt = 0; mt < MT; ++mt)
+                fa[mt] = -s.u.pipe.a[st][kk * 4 + q][wrow + mt * 8 + g];
 #pragma unroll
-              for (int nt = 0; nt < 4; ++nt) {
-                dmma(acc[0][nt], a0, b[nt]);
-                dmma(acc[1][nt], a1, b[nt]);
-              }
+              for (int nt = 0; nt < NT; ++nt)
+                fb[nt] = s.u.pipe.b[st][kk * 4 + q][wcol + nt * 8 + g];
+#pragma unroll
+              for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+                for (int nt = 0; nt < NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
             }
           }
         }
@@ -316,34 +541,21 @@ VB_DEVINL void potrf_big_matrix(BigSmem& s, double* __restrict__ A, int n, int l
       }
       __syncthreads();  // pipeline buffers are free: reuse as the C tile
 #pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
+      for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-          const int r = warp * 16 + mt * 8 + g, c = nt * 8 + 2 * q;
+        for (int nt = 0; nt < NT; ++nt) {
+          const int r = wrow + mt * 8 + g, c = wcol + nt * 8 + 2 * q;
           s.u.e.tile[c][r] = acc[mt][nt][0];
           s.u.e.tile[c + 1][r] = acc[mt][nt][1];
         }
       __syncthreads();
       if (first) {
         const bool below = r0 + nb < n;
-        if (warp == 0) {
-          double a[NB];
-#pragma unroll
-          for (int c = 0; c < NB; ++c) a[c] = s.u.e.tile[c][lane];
-          const int info = potf2_regs_warp<NB>(a, nb, lane, s.wbuf, s.sv, s.tv);
-          // store the factored diagonal block (lower part; on failure incl. the pivot)
-          double* Ad = A + (size_t)j0 * ld + j0;
-          const int ncol = info ? info : nb;
-#pragma unroll
-          for (int c = 0; c < NB; ++c)
-            if (c < ncol && lane >= c && lane < nb) {
-              s.u.e.tile[c][lane] = a[c];
-              Ad[(size_t)c * ld + lane] = a[c];
-            }
-          __syncwarp();
-          if (!info && below) trtri32_dmma_warp(&s.u.e.tile[0][0], LDA_S, s.tv, &s.inv[0][0], LDI,
-                                                s.u.e.scratch, lane);
-          if (lane == 0) s.info = info;
+        double* Ad = A + (size_t)j0 * ld + j0;
+        if constexpr (NB == 32) {
+          if (warp == 0) diag_block32(s, nb, lane, Ad, ld, below);
+        } else {
+          if (warp < 4) diag_block64(s, nb, warp, lane, Ad, ld, below);
         }
         __syncthreads();
         if (s.info) {
@@ -352,39 +564,14 @@ VB_DEVINL void potrf_big_matrix(BigSmem& s, double* __restrict__ A, int n, int l
         }
         if (!below) continue;  // no rows below the diagonal block in this pass
       }
-      // ---- panel factorize (TRSM): X = C inv(L11)^T on DMMA
-      double x[2][4][2];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) x[mt][nt][0] = x[mt][nt][1] = 0.0;
-      if (warp_active) {
-#pragma unroll
-        for (int k4 = 0; k4 < NB / 4; ++k4) {
-          const double a0 = s.u.e.tile[k4 * 4 + q][warp * 16 + g];
-          const double a1 = s.u.e.tile[k4 * 4 + q][warp * 16 + 8 + g];
-          double b[4];
-#pragma unroll
-          for (int nt = 0; nt < 4; ++nt) b[nt] = s.inv[k4 * 4 + q][nt * 8 + g];
-#pragma unroll
-          for (int nt = 0; nt < 4; ++nt) {
-            dmma(x[0][nt], a0, b[nt]);
-            dmma(x[1][nt], a1, b[nt]);
-          }
-        }
-      }
-      __syncthreads();
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-          const int r = warp * 16 + mt * 8 + g, c = nt * 8 + 2 * q;
-          s.u.e.tile[c][r] = x[mt][nt][0];
-          s.u.e.tile[c + 1][r] = x[mt][nt][1];
-        }
+      // ---- panel factorize (TRSM) on DMMA, 32 columns at a time with 32x32 inverses:
+      //      X1 = C1 inv(L11)^T;  [NB=64: C2 -= X1 L21^T;  X2 = C2 inv(L22)^T]
+      //      Each warp owns 16 rows of the tile (reads and writes only its rows), so no CTA
+      //      barrier is needed between the steps.
+      trsm_rows16<C>(s, warp, lane, r0 + warp * 16 < n);
       __syncthreads();
       const int row_lo = first ? j0 + nb : r0;
-      for (int idx = tid; idx < NB * MB; idx += kThreads) {
+      for (int idx = tid; idx < NB * MB; idx += C::THREADS) {
         const int c = idx / MB, r = idx % MB;
         const int row = r0 + r;
         if (c < nb && row < n && row >= row_lo) A[(size_t)(j0 + c) * ld + row] = s.u.e.tile[c][r];
@@ -394,28 +581,31 @@ VB_DEVINL void potrf_big_matrix(BigSmem& s, double* __restrict__ A, int n, int l
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 3)
+// range: 0 (NB = 64) or 1 (NB = 32). wait_upstream: the kernel directly follows the scan.
+template <class C>
+__global__ void __launch_bounds__(C::THREADS, C::MINB)
     potrf_blocked_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                         const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order) {
+                         const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
+                         int wait_upstream) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  BigSmem& s = *reinterpret_cast<BigSmem*>(smem_raw);
+  BlockedSmem<C>& s = *reinterpret_cast<BlockedSmem<C>*>(smem_raw);
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  pdl_wait();  // the scan's outputs (order, ctrl, info) are complete and visible
-  const int count_big = ctrl->count_big;
+  if (wait_upstream) pdl_wait();  // the scan's outputs (order, ctrl, info) are visible
+  pdl_launch_dependents();        // the next range's kernel may start filling freed SMs
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
   const int tid = threadIdx.x;
   for (;;) {
-    if (tid == 0) s.item = atomicAdd(&ctrl->head_big, 1);
+    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
     __syncthreads();
     const int it = s.item;
     __syncthreads();
-    if (it >= count_big) break;
-    const int m = order[it];
-    potrf_big_matrix(s, dA[m], d_n[m], d_ldda[m], d_info + m);
+    if (it >= count) break;
+    const int m = order[start + it];
+    potrf_blocked_matrix<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m);
     __syncthreads();
   }
-  // work list empty: let the warp-path kernel start on this SM
-  pdl_launch_dependents();
 }
 
 // ---------------------------------------------------------------------------------------
@@ -445,8 +635,8 @@ VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* inf
 
 // Warp path: one matrix (n <= 32) per warp, whole matrix in registers.
 // wait_upstream: 1 when launched directly after the scan (the only factorisation kernel),
-// 0 when launched after potrf_blocked_kernel (whose CTAs passed the scan's completion
-// before releasing this grid, so the scan's outputs are already visible).
+// 0 when launched after a blocked kernel (whose CTAs passed the scan's completion before
+// releasing this grid, so the scan's outputs are already visible).
 __global__ void __launch_bounds__(32 * kWarpsPerCta)
     potrf_warp_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                       const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -455,15 +645,15 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
   __shared__ WarpSmem s;
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
   if (wait_upstream) pdl_wait();
-  const int count_big = *(volatile const int*)&ctrl->count_big;
-  const int count_warp = *(volatile const int*)&ctrl->count_warp;
+  const int start = *(volatile const int*)&ctrl->start[2];
+  const int count = *(volatile const int*)&ctrl->count[2];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   for (;;) {
     int w = 0;
-    if (lane == 0) w = atomicAdd(&ctrl->head_warp, 1);
+    if (lane == 0) w = atomicAdd(&ctrl->head[2], 1);
     w = __shfl_sync(kFull, w, 0);
-    if (w >= count_warp) break;
-    const int m = order[count_big + w];
+    if (w >= count) break;
+    const int m = order[start + w];
     const int n = d_n[m], ld = d_ldda[m];
     if (n <= 8)
       potrf_warp_matrix<8>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
@@ -474,23 +664,44 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
   }
 }
 
+// ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
-static int g_occ_big = 0;
+static int g_occ32 = 0, g_occ64 = 0;
+static int g_t64 = -1;
+
+int potrf_t64() {
+  if (g_t64 < 0) {
+    const char* e = getenv("VB_T64");
+    g_t64 = e ? atoi(e) : 384;
+    if (g_t64 < kWarpMaxN) g_t64 = kWarpMaxN;
+  }
+  return g_t64;
+}
+
+template <class C>
+static cudaError_t setup_kernel(int* occ) {
+  cudaError_t e = cudaFuncSetAttribute(potrf_blocked_kernel<C>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)sizeof(BlockedSmem<C>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked_kernel<C>, C::THREADS,
+                                                    sizeof(BlockedSmem<C>));
+  if (*occ < 1) *occ = 1;
+  return e;
+}
 
 static cudaError_t init_device_info() {
   if (g_num_sms) return cudaSuccess;
   int dev;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+  int sms = 0;
+  e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(potrf_blocked_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)sizeof(BigSmem));
-  if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_big, potrf_blocked_kernel, kThreads,
-                                                    sizeof(BigSmem));
-  if (e != cudaSuccess) return e;
-  if (g_occ_big < 1) g_occ_big = 1;
+  if ((e = setup_kernel<Cfg32>(&g_occ32)) != cudaSuccess) return e;
+  if ((e = setup_kernel<Cfg64>(&g_occ64)) != cudaSuccess) return e;
+  potrf_t64();
+  g_num_sms = sms;
   return cudaSuccess;
 }
 
@@ -506,21 +717,36 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   cfg.stream = stream;
-  const bool big = max_n_hint > kWarpMaxN;
-  if (big) {
-    cfg.blockDim = dim3(kThreads);
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_big)));
-    cfg.dynamicSmemBytes = sizeof(BigSmem);
-    e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel, d_n, dA, d_ldda, d_info, ctrl, order);
+  int wait = 1;  // the first factorisation kernel after the scan waits for it
+  if (max_n_hint > g_t64) {
+    cfg.blockDim = dim3(Cfg64::THREADS);
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
+    cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg64>);
+    e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg64>, d_n, dA, d_ldda, d_info, ctrl, order,
+                           0, wait);
     if (e != cudaSuccess) return e;
+    wait = 0;
+  }
+  if (max_n_hint > kWarpMaxN) {
+    cfg.blockDim = dim3(Cfg32::THREADS);
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ32)));
+    cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg32>);
+    e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg32>, d_n, dA, d_ldda, d_info, ctrl, order,
+                           1, wait);
+    if (e != cudaSuccess) return e;
+    wait = 0;
   }
   const int warps = std::max(1, batch);
   cfg.blockDim = dim3(32 * kWarpsPerCta);
   cfg.gridDim = dim3(std::max(1, std::min((warps + kWarpsPerCta - 1) / kWarpsPerCta,
                                           g_num_sms * 8)));
   cfg.dynamicSmemBytes = 0;
-  return cudaLaunchKernelEx(&cfg, potrf_warp_kernel, d_n, dA, d_ldda, d_info, ctrl, order,
-                            big ? 0 : 1);
+  return cudaLaunchKernelEx(&cfg, potrf_warp_kernel, d_n, dA, d_ldda, d_info, ctrl, order, wait);
+}
+
+int potrf_num_launches(int max_n_hint) {
+  init_device_info();
+  return 1 + (max_n_hint > kWarpMaxN ? 1 : 0) + (max_n_hint > g_t64 ? 1 : 0);
 }
 
 }  // namespace vb

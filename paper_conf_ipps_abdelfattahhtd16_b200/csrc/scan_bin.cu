@@ -20,7 +20,7 @@ constexpr int kKeys = 4096;  // sort keys: min(n, kKeys-1) (larger n share the t
 
 __global__ void __launch_bounds__(kScanThreads, 1)
     scan_bin_kernel(const int* __restrict__ d_n, const int* __restrict__ d_ldda,
-                    int* __restrict__ d_info, int batch, int max_n, int check_max,
+                    int* __restrict__ d_info, int batch, int max_n, int check_max, int t64,
                     Ctrl* __restrict__ ctrl, int* __restrict__ order) {
   // Let the dependent (factorisation) grid launch and reach its griddepcontrol.wait now.
   pdl_launch_dependents();
@@ -86,15 +86,18 @@ __global__ void __launch_bounds__(kScanThreads, 1)
   }
   __syncthreads();
   if (tid == 0) {
-    // items with key > kWarpMaxN come first; start[kWarpMaxN] = their count.
-    const int count_big = hist[kWarpMaxN];
-    ctrl->head_big = 0;
-    ctrl->head_warp = 0;
-    ctrl->count_big = count_big;
+    // start[k] = #items with key > k (descending order): the three ranges are contiguous.
+    const int tk = t64 < kKeys - 1 ? (t64 > kWarpMaxN ? t64 : kWarpMaxN) : kKeys - 1;
+    const int c0 = hist[tk], c01 = hist[kWarpMaxN], call = hist[0];
+    ctrl->head[0] = ctrl->head[1] = ctrl->head[2] = 0;
+    ctrl->start[0] = 0;
+    ctrl->count[0] = c0;
+    ctrl->start[1] = c0;
+    ctrl->count[1] = c01 - c0;
+    ctrl->start[2] = c01;
+    ctrl->count[2] = call - c01;
     ctrl->max_n = wmax[0];
   }
-  // total valid = start[0] (key 0 is never used: n >= 1) -> count_warp = start[0]-count_big
-  if (tid == 1) ctrl->count_warp = hist[0] - hist[kWarpMaxN];
   __syncthreads();
   for (int i = tid; i < batch; i += kScanThreads) {
     const int n = d_n[i];
@@ -109,7 +112,7 @@ __global__ void __launch_bounds__(kScanThreads, 1)
 cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
                             bool check_max, Ctrl* ctrl, int* order, cudaStream_t stream) {
   scan_bin_kernel<<<1, kScanThreads, 0, stream>>>(d_n, d_ldda, d_info, batch, max_n,
-                                                  check_max ? 1 : 0, ctrl, order);
+                                                  check_max ? 1 : 0, potrf_t64(), ctrl, order);
   return cudaGetLastError();
 }
 
