@@ -49,7 +49,7 @@ struct BlockedCfg {
   static constexpr int LDI = NB + 4;
 };
 using Cfg32 = BlockedCfg<32, 128, 8, 1, 16, 3, 3>;
-using Cfg64 = BlockedCfg<64, 128, 4, 2, 16, 2, 2>;
+using Cfg64 = BlockedCfg<64, 128, 4, 2, 16, 3, 2>;
 
 constexpr int LDS_T = 20;  // TRTRI32 scratch leading dim
 
@@ -69,6 +69,9 @@ struct BlockedSmem {
     } e;
   } u;
   double inv[C::NB][C::LDI];  // inv[k][n] = (L11^-1)[n][k]  (DMMA B operand of the TRSM)
+  uint64_t full[C::STAGES];   // TMA ring: stage filled (producer arrive.expect_tx + bytes)
+  uint64_t empty[C::STAGES];  // TMA ring: stage consumed (one arrive per warp)
+  uint32_t chunks;            // chunks issued so far by this CTA (ring position)
   int item;
   int info;
 };
@@ -478,6 +481,51 @@ VB_DEVINL void trsm_rows16(BlockedSmem<C>& s, int warp, int lane, bool active) {
   }
 }
 
+// Issue chunk kc (global ring index gi) with TMA bulk copies, by warp 0: lanes 0..KC-1
+// copy A column segments (rows r0..r0+ra-1), lanes 16..16+KC-1 the panel rows j0..j0+rb-1.
+// Segment lengths are rounded up to an even row count (16-byte multiple); the extra row is
+// padding (ldda even and > n when n is odd). Rows beyond are stale and only ever feed
+// output rows/columns that are never stored.
+template <class C>
+VB_DEVINL void issue_stage_bulk(BlockedSmem<C>& s, uint32_t gi, int kc, const double* A, int n,
+                                int ld, int r0, int j0, int lane) {
+  static_assert(C::KC <= 16, "one lane per column segment");
+  const int st = gi % C::STAGES;
+  const uint32_t u = gi / C::STAGES;
+  const int ra = (min(C::MB, n - r0) + 1) & ~1;
+  const int rb = (min(C::NB, n - j0) + 1) & ~1;
+  if (lane == 0) {
+    if (u > 0) mbar_wait(&s.empty[st], (u - 1) & 1);
+    mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * 8));
+  }
+  __syncwarp();
+  const int k0 = kc * C::KC;
+  if (lane < C::KC) {
+    bulk_g2s(&s.u.pipe.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * 8, &s.full[st]);
+  } else if (lane >= 16 && lane < 16 + C::KC) {
+    const int c = lane - 16;
+    bulk_g2s(&s.u.pipe.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * 8, &s.full[st]);
+  }
+}
+
+// One k-chunk of the panel update for this warp's tile: acc -= A_chunk B_chunk^T.
+template <class C>
+VB_DEVINL void mma_chunk(BlockedSmem<C>& s, int st, double (&acc)[C::MT][C::NT][2], int wrow,
+                         int wcol, int g, int q) {
+#pragma unroll
+  for (int kk = 0; kk < C::KC / 4; ++kk) {
+    double fa[C::MT], fb[C::NT];
+#pragma unroll
+    for (int mt = 0; mt < C::MT; ++mt) fa[mt] = -s.u.pipe.a[st][kk * 4 + q][wrow + mt * 8 + g];
+#pragma unroll
+    for (int nt = 0; nt < C::NT; ++nt) fb[nt] = s.u.pipe.b[st][kk * 4 + q][wcol + nt * 8 + g];
+#pragma unroll
+    for (int mt = 0; mt < C::MT; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < C::NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+  }
+}
+
 // Blocked left-looking Cholesky of one matrix by the whole CTA.
 template <class C>
 VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, int n, int ld,
@@ -488,6 +536,8 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
   const int g = lane >> 2, q = lane & 3;
   const int wrow = (warp % C::WARPS_M) * C::WM;  // warp's first row within the block
   const int wcol = (warp / C::WARPS_M) * C::WN;  // warp's first panel column
+  // TMA bulk copies need 16-byte aligned column segments: even ldda and aligned base.
+  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
   for (int j0 = 0; j0 < n; j0 += NB) {
     const int nb = min(NB, n - j0);
     const int nk = j0 / KC;
@@ -508,36 +558,44 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
           }
       // ---- panel update on DMMA: acc -= L[r0:r0+MB, 0:j0] L[j0:j0+NB, 0:j0]^T
       if (nk > 0) {
-#pragma unroll
-        for (int st = 0; st < STAGES - 1; ++st) {
-          if (st < nk) load_stage<C>(s, st, st, A, n, ld, r0, j0);
-          cp_async_commit();
-        }
-        for (int kc = 0; kc < nk; ++kc) {
-          cp_async_wait<STAGES - 2>();
-          __syncthreads();
-          const int pf = kc + STAGES - 1;
-          if (pf < nk) load_stage<C>(s, pf % STAGES, pf, A, n, ld, r0, j0);
-          cp_async_commit();
-          const int st = kc % STAGES;
-          if (warp_active) {
-#pragma unroll
-            for (int kk = 0; kk < KC / 4; ++kk) {
-              double fa[MT], fb[NT];
-#pragma unroll
-              for (int mt = 0; mt < MT; ++mt)
-                fa[mt] = -s.u.pipe.a[st][kk * 4 + q][wrow + mt * 8 + g];
-#pragma unroll
-              for (int nt = 0; nt < NT; ++nt)
-                fb[nt] = s.u.pipe.b[st][kk * 4 + q][wcol + nt * 8 + g];
-#pragma unroll
-              for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-                for (int nt = 0; nt < NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
-            }
+        if (bulk) {
+          // TMA ring: warp 0 issues 1-D bulk copies of whole column segments into stage
+          // (chunk % STAGES); consumers wait on full[], release with one arrive per warp on
+          // empty[]; the producer waits on empty[] before refilling a stage.
+          const uint32_t gb = s.chunks;
+          if (warp == 0) {
+            fence_proxy_async();  // generic smem accesses (epilogue) before async writes
+            for (int p = 0; p < STAGES - 1 && p < nk; ++p)
+              issue_stage_bulk<C>(s, gb + p, p, A, n, ld, r0, j0, lane);
           }
+          for (int kc = 0; kc < nk; ++kc) {
+            const uint32_t gi = gb + kc;
+            const int st = gi % STAGES;
+            if (warp == 0 && kc + STAGES - 1 < nk)
+              issue_stage_bulk<C>(s, gi + STAGES - 1, kc + STAGES - 1, A, n, ld, r0, j0, lane);
+            mbar_wait(&s.full[st], (gi / STAGES) & 1);
+            if (warp_active) mma_chunk<C>(s, st, acc, wrow, wcol, g, q);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&s.empty[st]);
+          }
+          __syncthreads();
+          if (tid == 0) s.chunks = gb + nk;
+        } else {
+#pragma unroll
+          for (int st = 0; st < STAGES - 1; ++st) {
+            if (st < nk) load_stage<C>(s, st, st, A, n, ld, r0, j0);
+            cp_async_commit();
+          }
+          for (int kc = 0; kc < nk; ++kc) {
+            cp_async_wait<STAGES - 2>();
+            __syncthreads();
+            const int pf = kc + STAGES - 1;
+            if (pf < nk) load_stage<C>(s, pf % STAGES, pf, A, n, ld, r0, j0);
+            cp_async_commit();
+            if (warp_active) mma_chunk<C>(s, kc % STAGES, acc, wrow, wcol, g, q);
+          }
+          cp_async_wait<0>();
         }
-        cp_async_wait<0>();
       }
       __syncthreads();  // pipeline buffers are free: reuse as the C tile
 #pragma unroll
@@ -557,6 +615,7 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
         } else {
           if (warp < 4) diag_block64(s, nb, warp, lane, Ad, ld, below);
         }
+        fence_proxy_async();  // generic smem writes before the next TMA refill of this memory
         __syncthreads();
         if (s.info) {
           if (tid == 0) *info_out = j0 + s.info;
@@ -568,7 +627,8 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
       //      X1 = C1 inv(L11)^T;  [NB=64: C2 -= X1 L21^T;  X2 = C2 inv(L22)^T]
       //      Each warp owns 16 rows of the tile (reads and writes only its rows), so no CTA
       //      barrier is needed between the steps.
-      trsm_rows16<C>(s, warp, lane, r0 + warp * 16 < n);
+      trsm_rows16<C>(s, warp, lane,
+                     r0 + warp * 16 < n && !(first && warp * 16 + 16 <= nb));
       __syncthreads();
       const int row_lo = first ? j0 + nb : r0;
       for (int idx = tid; idx < NB * MB; idx += C::THREADS) {
@@ -576,6 +636,7 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
         const int row = r0 + r;
         if (c < nb && row < n && row >= row_lo) A[(size_t)(j0 + c) * ld + row] = s.u.e.tile[c][r];
       }
+      fence_proxy_async();  // generic smem accesses before the next TMA refill of this memory
       __syncthreads();
     }
   }
@@ -591,6 +652,15 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
   extern __shared__ __align__(16) unsigned char smem_raw[];
   BlockedSmem<C>& s = *reinterpret_cast<BlockedSmem<C>*>(smem_raw);
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < C::STAGES; ++i) {
+      mbar_init(&s.full[i], 1);
+      mbar_init(&s.empty[i], C::THREADS / 32);
+    }
+    s.chunks = 0;
+    fence_proxy_async();  // make the initialised barriers visible to the async proxy
+  }
+  __syncthreads();
   if (wait_upstream) pdl_wait();  // the scan's outputs (order, ctrl, info) are visible
   pdl_launch_dependents();        // the next range's kernel may start filling freed SMs
   const int count = *(volatile const int*)&ctrl->count[range];
@@ -672,7 +742,7 @@ static int g_t64 = -1;
 int potrf_t64() {
   if (g_t64 < 0) {
     const char* e = getenv("VB_T64");
-    g_t64 = e ? atoi(e) : 384;
+    g_t64 = e ? atoi(e) : 512;
     if (g_t64 < kWarpMaxN) g_t64 = kWarpMaxN;
   }
   return g_t64;
