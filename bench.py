@@ -230,12 +230,8 @@ def our_arm(args, cfg, rank, world, local_rank):
     n_all = vbgen.sizes(cfg)
     if args.batch_limit:
         n_all = n_all[: args.batch_limit]
-    gidx_all = np.arange(len(n_all), dtype=np.int32)
-    if world > 1:
-        owner = vb.vbatched_partition_lpt(n_all, world)
-        mine = gidx_all[owner == rank]
-    else:
-        mine = gidx_all
+    from paper_conf_ipps_abdelfattahhtd16_b200 import shard
+    mine = shard.shard_indices(n_all, world, rank)  # LPT on n^3/3, identical on every rank
     n_loc = n_all[mine]
     db = DeviceBatch(n_loc, seed=cfg.seed, gidx=mine, nonspd_mod=cfg.nonspd_mod, device=dev)
     ws = torch.empty(vb.vbatched_dpotrf_workspace_size(db.B), dtype=torch.uint8, device=dev)
@@ -279,17 +275,17 @@ def our_arm(args, cfg, rank, world, local_rank):
     info = db.info()
     ok_local = vbgen.expected_flops(n_loc[info == 0])
     alg_bytes_local = vbgen.algorithmic_bytes(n_loc[info == 0])
-    bad_info = int(np.sum(info != expected_info(cfg, n_loc, mine)))
-    loc = torch.tensor([sum(step_ms), sum(kern_ms), ok_local, alg_bytes_local, bad_info],
-                       dtype=torch.float64, device=dev)
+    # global info[] from every rank's (index, info) pairs; flops count only info == 0 matrices
+    info_all = shard.gather_info(len(n_all), mine, info, device=dev)
+    bad_info = int(np.sum(info_all != expected_info(cfg, n_all, np.arange(len(n_all)))))
+    max_total_ms = shard.max_over_ranks(sum(step_ms), device=dev)
+    flops_total = vbgen.expected_flops(n_all[info_all == 0])
+    per_rank_ms = [sum(step_ms) / args.steps]
     if world > 1:
-        allv = [torch.zeros_like(loc) for _ in range(world)]
-        dist.all_gather(allv, loc)
-        allv = torch.stack(allv).cpu().numpy()
-    else:
-        allv = loc.cpu().numpy()[None, :]
-    max_total_ms = float(allv[:, 0].max())
-    flops_total = float(allv[:, 2].sum())
+        t = torch.tensor([sum(step_ms) / args.steps], dtype=torch.float64, device=dev)
+        allt = [torch.zeros_like(t) for _ in range(world)]
+        dist.all_gather(allt, t)
+        per_rank_ms = [float(x.item()) for x in allt]
     value = flops_total * args.steps / (max_total_ms / 1e3) / 1e9
 
     # roofline of the dominant kernel (potrf_persistent_kernel) on this rank
@@ -334,8 +330,8 @@ def our_arm(args, cfg, rank, world, local_rank):
             "data": "synthetic", "config": config_dict(cfg, world),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches_per_step * args.steps, "clocks": clocks,
-            "info_mismatches": int(allv[:, 4].sum()),
-            "per_rank_ms": [float(x) / args.steps for x in allv[:, 0]],
+            "info_mismatches": bad_info,
+            "per_rank_ms": per_rank_ms,
             "library": vb.vbatched_version(),
         }
         if args.batch_limit:

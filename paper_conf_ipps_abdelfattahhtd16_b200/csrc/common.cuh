@@ -89,6 +89,11 @@ VB_DEVINL void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* 
 }
 // Order this thread's prior generic-proxy shared-memory accesses before later async-proxy ones.
 VB_DEVINL void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
+// Same for global memory: this thread's generic stores (the L panels it wrote) before later
+// TMA (async-proxy) reads of them by any thread of the CTA (after a barrier).
+VB_DEVINL void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;\n" ::: "memory");
+}
 
 // Programmatic dependent launch (PDL): wait for the upstream grid's results / let the
 // downstream grid start its prologue early.

@@ -615,7 +615,8 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
         } else {
           if (warp < 4) diag_block64(s, nb, warp, lane, Ad, ld, below);
         }
-        fence_proxy_async();  // generic smem writes before the next TMA refill of this memory
+        fence_proxy_async();         // generic smem writes before the next TMA refill
+        fence_proxy_async_global();  // L11 stores before later TMA reads of them
         __syncthreads();
         if (s.info) {
           if (tid == 0) *info_out = j0 + s.info;
@@ -636,7 +637,8 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
         const int row = r0 + r;
         if (c < nb && row < n && row >= row_lo) A[(size_t)(j0 + c) * ld + row] = s.u.e.tile[c][r];
       }
-      fence_proxy_async();  // generic smem accesses before the next TMA refill of this memory
+      fence_proxy_async();         // generic smem accesses before the next TMA refill
+      fence_proxy_async_global();  // this panel's L stores before later TMA reads of them
       __syncthreads();
     }
   }
