@@ -87,6 +87,18 @@ VB_DEVINL void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* 
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// L2 prefetch of a contiguous global range (TMA unit; 16-byte aligned, size multiple of 16).
+VB_DEVINL void bulk_prefetch_l2(const void* gsrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(gsrc), "r"(bytes) : "memory");
+}
+// C-fragment -> A-fragment of m8n8k4 DMMA: this lane's C values (row g, cols 2q, 2q+1) of an
+// 8x8 tile; returns A[g][4*half + q] for the k-step covering tile columns 4*half..4*half+3.
+VB_DEVINL double cfrag_to_afrag(double c0, double c1, int half, int lane) {
+  const int src = (lane & ~3) | (2 * half + ((lane & 3) >> 1));
+  const double v0 = __shfl_sync(0xffffffffu, c0, src);
+  const double v1 = __shfl_sync(0xffffffffu, c1, src);
+  return (lane & 1) ? v1 : v0;
+}
 // Order this thread's prior generic-proxy shared-memory accesses before later async-proxy ones.
 VB_DEVINL void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
 // Same for global memory: this thread's generic stores (the L panels it wrote) before later

@@ -37,6 +37,18 @@
 
 namespace vb {
 
+// Optional phase timers (debug builds with -DVB_PHASE_PROF): warp 0 lane 0 of each CTA of the
+// v2 kernel accumulates clock64() cycles per phase; read with vbatched_debug_phases().
+#ifdef VB_PHASE_PROF
+__device__ unsigned long long g_phase[8];
+#define VB_T0(v) long long v = clock64();
+#define VB_ADD(i, v) \
+  if (threadIdx.x == 0) atomicAdd(&g_phase[i], (unsigned long long)(clock64() - (v)));
+#else
+#define VB_T0(v)
+#define VB_ADD(i, v)
+#endif
+
 template <int NB_, int MB_, int WARPS_M_, int WARPS_N_, int KC_, int STAGES_, int MINB_>
 struct BlockedCfg {
   static constexpr int NB = NB_, MB = MB_, WARPS_M = WARPS_M_, WARPS_N = WARPS_N_;
@@ -51,7 +63,7 @@ struct BlockedCfg {
 using Cfg32 = BlockedCfg<32, 128, 8, 1, 16, 3, 3>;
 using Cfg64 = BlockedCfg<64, 128, 4, 2, 16, 3, 2>;
 
-constexpr int LDS_T = 20;  // TRTRI32 scratch leading dim
+constexpr int LDS_T = 18;  // TRTRI32 scratch leading dim (16 columns used)
 
 template <class C>
 struct BlockedSmem {
@@ -62,7 +74,7 @@ struct BlockedSmem {
     } pipe;
     struct {
       double tile[C::NB][C::LDA];  // C tile: [col][row], aliases the pipeline after the k loop
-      double scratch[16 * LDS_T * 2];  // TRTRI32 scratch
+      double scratch[16 * LDS_T];  // TRTRI32 scratch
       double wbuf[64];
       double sv[C::NB];
       double tv[C::NB];
@@ -680,6 +692,413 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
   }
 }
 
+// =======================================================================================
+// v2 blocked kernel (large n): warp w owns 16 full rows of each 128-row block, so the TRSM
+// runs from registers and stores straight to global; the TMA stage ring is not aliased
+// with anything, so the producer (warp 0) keeps prefetching across the row blocks of a
+// panel; CTA-wide barriers only around the diagonal block and at the panel end.
+template <int NB_, int KC_, int STAGES_, int MINB_>
+struct Cfg2 {
+  static constexpr int NB = NB_, KC = KC_, STAGES = STAGES_, MINB = MINB_;
+  static constexpr int WARPS = 8, THREADS = 256, MB = 128, NT = NB / 8;
+  static constexpr int LDA = MB + 4, LDB = NB + 4, LDT = NB + 4;
+};
+using Cfg64b = Cfg2<64, 16, 3, 2>;
+
+template <class C>
+struct Smem2 {
+  double a[C::STAGES][C::KC][C::LDA];  // A chunk: [k][row]
+  double b[C::STAGES][C::KC][C::LDB];  // B chunk: [k][panel row]
+  // Diagonal block T[c][r]. After diag_block64v2: T11 slot = inv(L22) as B operand,
+  // T12 slot (cols 32..63, rows 0..31) = inv(L11) as B operand, T21 = L21, T22 = L22.
+  double T[C::NB][C::LDT];
+  double S[16 * LDS_T];  // TRTRI scratch
+  double wbuf[64];
+  double sv[C::NB];
+  double tv[C::NB];
+  uint64_t full[C::STAGES];
+  uint64_t empty[C::STAGES];
+  uint32_t chunks;  // chunks issued so far (ring position)
+  int item;
+  int info;
+};
+
+// Diagonal 64x64 block by warps 0..3 (named barrier 1): L11 = potf2(C11), inv(L11) -> T12,
+// L21 = C21 inv(L11)^T -> T21, C22 -= L21 L21^T, L22 = potf2(C22), inv(L22) -> T11.
+// Stores L11, L21, L22 (rows < nb) to global (Ad, ld). Sets s.info (1-based, in-block).
+__device__ __noinline__ void diag_block64v2(Smem2<Cfg64b>& s, int nb, int wg, int lane,
+                                            double* Ad, int ld, bool below) {
+  constexpr int LDT = Cfg64b::LDT;
+  double* T = &s.T[0][0];
+  double* INV11 = T + 32 * LDT;  // T12 slot: INV11[k*LDT + n]
+  double* INV22 = T;             // T11 slot (after L11 is dead)
+  const int g = lane >> 2, q = lane & 3;
+  const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
+  const int nb1 = min(nb, 32), nb2 = nb - nb1;
+  if (wg == 0) {
+    const int info = potf2_block32(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
+    if (!info && nb2 > 0) trtri32_dmma_warp(T, LDT, s.tv, INV11, LDT, s.S, LDS_T, lane);
+    if (lane == 0) s.info = info;
+  }
+  bar_group(1, 128);
+  if (s.info || nb2 == 0) return;
+  {  // L21 = C21 inv(L11)^T
+    double acc[2][2][2] = {};
+    mm32_quarter(acc, wg, lane, [&](int m, int k) { return T[k * LDT + 32 + m]; },
+                 [&](int k, int n) { return INV11[k * LDT + n]; });
+    bar_group(1, 128);
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
+          T[c * LDT + r] = acc[mt][nt][h];
+          if (r < nb) Ad[(size_t)c * ld + r] = acc[mt][nt][h];
+        }
+  }
+  bar_group(1, 128);
+  {  // C22 -= L21 L21^T
+    double acc[2][2][2];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          acc[mt][nt][h] = T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g];
+    mm32_quarter(acc, wg, lane, [&](int m, int k) { return -T[k * LDT + 32 + m]; },
+                 [&](int k, int n) { return T[k * LDT + 32 + n]; });
+    bar_group(1, 128);
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
+  }
+  bar_group(1, 128);
+  if (wg == 0) {
+    double* T22 = T + 32 * LDT + 32;
+    const int info = potf2_block32(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf,
+                                   s.sv + 32, s.tv + 32);
+    if (!info && below) trtri32_dmma_warp(T22, LDT, s.tv + 32, INV22, LDT, s.S, LDS_T, lane);
+    if (lane == 0) s.info = info ? 32 + info : 0;
+  }
+  bar_group(1, 128);
+}
+
+// Producer (warp 0): chunk kc of the row block at r0 into ring slot gi % STAGES.
+template <class C>
+VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, int n, int ld,
+                            int r0, int j0, int lane, bool bulk) {
+  const int st = gi % C::STAGES;
+  const uint32_t u = gi / C::STAGES;
+  const int k0 = kc * C::KC;
+  if (lane == 0 && u > 0) mbar_wait(&s.empty[st], (u - 1) & 1);
+  __syncwarp();
+  if (bulk) {
+    const int ra = (min(C::MB, n - r0) + 1) & ~1;
+    const int rb = (min(C::NB, n - j0) + 1) & ~1;
+    if (lane == 0) mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * 8));
+    __syncwarp();
+    if (lane < C::KC) {
+      bulk_g2s(&s.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * 8, &s.full[st]);
+    } else if (lane >= 16 && lane < 16 + C::KC) {
+      const int c = lane - 16;
+      bulk_g2s(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * 8, &s.full[st]);
+    }
+  } else {  // odd ldda / unaligned base: plain loads by the producer warp, then arrive
+    const int ra = min(C::MB, n - r0), rb = min(C::NB, n - j0);
+    for (int c = 0; c < C::KC; ++c) {
+      const double* col = A + (size_t)(k0 + c) * ld;
+      for (int r = lane; r < ra; r += 32) s.a[st][c][r] = col[r0 + r];
+      for (int r = lane; r < rb; r += 32) s.b[st][c][r] = col[j0 + r];
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&s.full[st]);
+  }
+}
+
+// TRSM of this warp's 16 rows, in registers: X = C inv(L)^T (NB = 64: two 32-column steps
+// with inv(L11), L21, inv(L22) from s.T). Result overwrites acc.
+VB_DEVINL void trsm_regs64(Smem2<Cfg64b>& s, double (&acc)[2][8][2], int lane) {
+  constexpr int LDT = Cfg64b::LDT;
+  const double* T = &s.T[0][0];
+  const int g = lane >> 2, q = lane & 3;
+  double x[2][4][2];
+  // X1 = C1 inv(L11)^T: B[k][n] = INV11[k][n] = T[(32 + k)][n]
+#pragma unroll
+  for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) x[mt][nt][0] = x[mt][nt][1] = 0.0;
+#pragma unroll
+  for (int ks = 0; ks < 8; ++ks) {
+    double fa[2], fb[4];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+      fa[mt] = cfrag_to_afrag(acc[mt][ks >> 1][0], acc[mt][ks >> 1][1], ks & 1, lane);
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) fb[nt] = T[(32 + ks * 4 + q) * LDT + nt * 8 + g];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+  }
+  // C2 -= X1 L21^T: B[k][n] = L21[n][k] = T[k][32 + n]
+#pragma unroll
+  for (int ks = 0; ks < 8; ++ks) {
+    double fa[2], fb[4];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+      fa[mt] = -cfrag_to_afrag(x[mt][ks >> 1][0], x[mt][ks >> 1][1], ks & 1, lane);
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) fb[nt] = T[(ks * 4 + q) * LDT + 32 + nt * 8 + g];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][4 + nt], fa[mt], fb[nt]);
+  }
+#pragma unroll
+  for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) {
+      acc[mt][nt][0] = x[mt][nt][0];
+      acc[mt][nt][1] = x[mt][nt][1];
+      x[mt][nt][0] = x[mt][nt][1] = 0.0;
+    }
+  // X2 = C2 inv(L22)^T: B[k][n] = INV22[k][n] = T[k][n]
+#pragma unroll
+  for (int ks = 0; ks < 8; ++ks) {
+    double fa[2], fb[4];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+      fa[mt] = cfrag_to_afrag(acc[mt][4 + (ks >> 1)][0], acc[mt][4 + (ks >> 1)][1], ks & 1, lane);
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) fb[nt] = T[(ks * 4 + q) * LDT + nt * 8 + g];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+  }
+#pragma unroll
+  for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) {
+      acc[mt][4 + nt][0] = x[mt][nt][0];
+      acc[mt][4 + nt][1] = x[mt][nt][1];
+    }
+}
+
+template <class C>
+VB_DEVINL void potrf_blocked2_matrix(Smem2<C>& s, double* __restrict__ A, int n, int ld,
+                                     int* info_out) {
+  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  const int wrow = warp * 16;
+  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
+  uint32_t gcons = s.chunks;  // ring position of the next chunk to consume (all threads)
+  for (int j0 = 0; j0 < n; j0 += NB) {
+    const int nb = min(NB, n - j0);
+    const int nk = j0 / KC;
+    // producer state (meaningful in warp 0): next chunk of this panel to issue
+    int p_r0 = j0, p_kc = 0;
+    uint32_t gprod = gcons;
+    auto produce = [&]() {
+      if (p_r0 < n && nk > 0) {
+        issue_chunk2<C>(s, gprod, p_kc, A, n, ld, p_r0, j0, lane, bulk);
+        ++gprod;
+        if (++p_kc == nk) {
+          p_kc = 0;
+          p_r0 += MB;
+        }
+      }
+    };
+    if (warp == 0) {
+      fence_proxy_async();
+      for (int i = 0; i < STAGES - 1; ++i) produce();
+    }
+    for (int r0 = j0; r0 < n; r0 += MB) {
+      const bool first = (r0 == j0);
+      const bool active = (r0 + wrow) < n;
+      VB_T0(t_a)
+      double acc[2][NT][2];
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
+            const bool v = row < n && col < j0 + nb && row >= col;
+            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+          }
+      VB_ADD(5, t_a)
+      if (warp == 0 && lane < NB && bulk && r0 + MB < n) {
+        // warm L2 with the next row block's panel values (the accumulators' start)
+        const int rn = (min(MB, n - r0 - MB) + 1) & ~1;
+        if (lane < nb) bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0 + MB, rn * 8);
+      }
+      // columns this warp must compute: in the first row block the diagonal-block warps skip
+      // the tiles strictly above the diagonal (SYRK); warp-uniform bound
+#ifndef VB_V2_SKIP
+#define VB_V2_SKIP 0
+#endif
+      const int ntl = (VB_V2_SKIP && first && wrow < NB) ? (wrow + 16) / 8 : NT;
+      VB_T0(t_k)
+      for (int kc = 0; kc < nk; ++kc) {
+        if (warp == 0) produce();
+        const uint32_t gi = gcons + kc;
+        const int st = gi % STAGES;
+        mbar_wait(&s.full[st], (gi / STAGES) & 1);
+        if (active) {
+#pragma unroll
+          for (int kk = 0; kk < KC / 4; ++kk) {
+            double fa[2], fb[NT];
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+              for (int nt = 0; nt < NT; ++nt)
+                if (nt < ntl) dmma(acc[mt][nt], fa[mt], fb[nt]);
+          }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s.empty[st]);
+      }
+      gcons += nk;
+      VB_ADD(0, t_k)
+      VB_T0(t_d)
+      if (first) {
+        // Diagonal-block warps hand their accumulators to smem and factor the block; the
+        // other warps wait for inv(L) and do their TRSM. Two separate branches joined only by
+        // named barriers, so no accumulator is live across the out-of-line diagonal call.
+        const bool below = r0 + nb < n;
+        const bool diag_warp = warp < NB / 16;  // this warp's 16 rows are diagonal-block rows
+        bool failed;
+        if (diag_warp) {
+#pragma unroll
+          for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+              s.T[nt * 8 + 2 * q][wrow + mt * 8 + g] = acc[mt][nt][0];
+              s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
+            }
+          bar_group(2, C::THREADS);
+          diag_block64v2(s, nb, warp, lane, A + (size_t)j0 * ld + j0, ld, below);
+          bar_group(3, C::THREADS);
+          failed = s.info != 0;
+        } else {
+          bar_group(2, C::THREADS);
+          bar_group(3, C::THREADS);
+          failed = s.info != 0;
+          if (!failed && below && active) {
+            trsm_regs64(s, acc, lane);
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+              for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                  const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
+                  if (row < n && row >= j0 + nb && col < nb)
+                    A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+                }
+          }
+        }
+        VB_ADD(1, t_d)
+        if (failed) {
+          if (tid == 0) *info_out = j0 + s.info;
+          // consume the chunks the producer already issued for this panel so the ring stays
+          // consistent for the next matrix
+          if (warp == 0) {
+            for (uint32_t gi = gcons; gi < gprod; ++gi) {
+              const int st = gi % STAGES;
+              if (lane == 0) mbar_wait(&s.full[st], (gi / STAGES) & 1);
+            }
+          }
+          __syncthreads();
+          if (warp == 0 && lane == 0) {
+            for (uint32_t gi = gcons; gi < gprod; ++gi)
+              for (int w = 0; w < C::WARPS; ++w) mbar_arrive(&s.empty[gi % STAGES]);
+          }
+          const uint32_t done = __shfl_sync(kFull, gprod, 0);
+          if (tid == 0) s.chunks = done;
+          __syncthreads();
+          return;
+        }
+        continue;
+      }
+      VB_T0(t_t)
+      // ---- TRSM in registers + direct stores of the rows below the diagonal block
+      if (active) {
+        trsm_regs64(s, acc, lane);
+        const int row_lo = r0;
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
+              if (row < n && row >= row_lo && col < nb)
+                A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+            }
+      }
+      VB_ADD(2, t_t)
+    }
+    // panel end: every L value of this panel is stored before the next panel's TMA reads
+    VB_T0(t_p)
+    fence_proxy_async_global();
+    __syncthreads();
+    VB_ADD(3, t_p)
+  }
+  if (tid == 0) s.chunks = gcons;
+  __syncthreads();
+}
+
+template <class C>
+__global__ void __launch_bounds__(C::THREADS, C::MINB)
+    potrf_blocked2_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                          const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
+                          int range, int wait_upstream) {
+  extern __shared__ __align__(128) unsigned char smem_raw2[];
+  Smem2<C>& s = *reinterpret_cast<Smem2<C>*>(smem_raw2);
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < C::STAGES; ++i) {
+      mbar_init(&s.full[i], 1);
+      mbar_init(&s.empty[i], C::WARPS);
+    }
+    s.chunks = 0;
+    fence_proxy_async();
+  }
+  __syncthreads();
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int tid = threadIdx.x;
+  for (;;) {
+    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
+    __syncthreads();
+    const int it = s.item;
+    __syncthreads();
+    if (it >= count) break;
+    const int m = order[start + it];
+    VB_T0(t_m)
+    potrf_blocked2_matrix<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m);
+    VB_ADD(4, t_m)
+  }
+}
+
 // ---------------------------------------------------------------------------------------
 constexpr int kWarpsPerCta = 2;
 struct WarpSmem {
@@ -738,8 +1157,9 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 
 // ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
-static int g_occ32 = 0, g_occ64 = 0;
+static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0;
 static int g_t64 = -1;
+static int g_v2 = -1;
 
 int potrf_t64() {
   if (g_t64 < 0) {
@@ -772,6 +1192,17 @@ static cudaError_t init_device_info() {
   if (e != cudaSuccess) return e;
   if ((e = setup_kernel<Cfg32>(&g_occ32)) != cudaSuccess) return e;
   if ((e = setup_kernel<Cfg64>(&g_occ64)) != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(potrf_blocked2_kernel<Cfg64b>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64b>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64b, potrf_blocked2_kernel<Cfg64b>,
+                                                    Cfg64b::THREADS, sizeof(Smem2<Cfg64b>));
+  if (e != cudaSuccess) return e;
+  if (g_occ64b < 1) g_occ64b = 1;
+  {
+    const char* v = getenv("VB_V2");
+    g_v2 = v ? atoi(v) : 1;
+  }
   potrf_t64();
   g_num_sms = sms;
   return cudaSuccess;
@@ -791,11 +1222,19 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.stream = stream;
   int wait = 1;  // the first factorisation kernel after the scan waits for it
   if (max_n_hint > g_t64) {
-    cfg.blockDim = dim3(Cfg64::THREADS);
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
-    cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg64>);
-    e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg64>, d_n, dA, d_ldda, d_info, ctrl, order,
-                           0, wait);
+    if (g_v2) {
+      cfg.blockDim = dim3(Cfg64b::THREADS);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64b)));
+      cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64b>);
+      e = cudaLaunchKernelEx(&cfg, potrf_blocked2_kernel<Cfg64b>, d_n, dA, d_ldda, d_info, ctrl,
+                             order, 0, wait);
+    } else {
+      cfg.blockDim = dim3(Cfg64::THREADS);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
+      cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg64>);
+      e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg64>, d_n, dA, d_ldda, d_info, ctrl,
+                             order, 0, wait);
+    }
     if (e != cudaSuccess) return e;
     wait = 0;
   }
@@ -822,3 +1261,14 @@ int potrf_num_launches(int max_n_hint) {
 }
 
 }  // namespace vb
+
+#ifdef VB_PHASE_PROF
+extern "C" int vbatched_debug_phases(unsigned long long* out, int reset) {
+  cudaError_t e = cudaMemcpyFromSymbol(out, vb::g_phase, sizeof(unsigned long long) * 8);
+  if (reset) {
+    unsigned long long z[8] = {};
+    cudaMemcpyToSymbol(vb::g_phase, z, sizeof z);
+  }
+  return (int)e;
+}
+#endif

@@ -5,6 +5,8 @@ Gates (BASELINE.json north_star): info[] bit-exact; bac
 oracle's L <= 1e-10 (kappa <= 1e4). Exact integer families must be bit-exact. The strict
 upper triangle and padding rows must be bit-identical afterwards (NaN sentinels).
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -111,9 +113,50 @@ def test_nonspd_info_positions():
     _check_sentinels(db)
 
 
+@pytest.mark.parametrize("v2", ["1", "0"])
+def test_nonspd_large_and_ring_recovery(v2, monkeypatch):
+    """Failures inside the NB=64 kernel (n > 512): failing pivots in the first and second
+    32-column halves of a 64-wide diagonal block, at panel starts and at n; the TMA ring must
+    stay consistent for the matrices the same CTA factors afterwards (checked by parity of
+    healthy matrices in the same batch). VB_V2 selects the kernel variant (read at first use,
+    so each variant runs in a subprocess)."""
+    import subprocess
+    import sys
+    code = f"""
+import os, sys
+sys.path.insert(0, {repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))})
+import numpy as np, torch, vbgen
+from harness import DeviceBatch, compare_with_oracle
+cases = [(700, 1), (700, 33), (700, 64), (700, 65), (700, 129), (700, 700), (1024, 511),
+         (1024, 1024), (600, 0), (800, 0), (513, 513), (900, 0), (1000, 97)]
+n_arr = np.array([c[0] for c in cases], dtype=np.int32)
+db = DeviceBatch(n_arr, seed=8)
+inputs = {{}}
+for i, (n, k) in enumerate(cases):
+    A = vbgen.f1_matrix(8, i, n)
+    if k:
+        A[k - 1, k - 1] = -A[k - 1, k - 1]
+    inputs[i] = A
+    db.set_matrix(i, A)
+db.dpotrf()
+torch.cuda.synchronize()
+info = db.info()
+assert list(info) == [k for _, k in cases], (list(info), cases)
+for i in range(db.B):
+    r = compare_with_oracle(inputs[i], db.block(i), info[i])
+    assert r["ok"], (i, r)
+print("OK")
+"""
+    env = dict(os.environ, VB_V2=v2)
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env,
+                         timeout=600)
+    assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
+
+
 def test_nan_info():
     cases = [(8, (2, 2)), (8, (5, 1)), (40, (33, 33)), (40, (39, 10)), (100, (70, 64)),
-             (100, (0, 0)), (100, (99, 99))]
+             (100, (0, 0)), (100, (99, 99)), (700, (40, 40)), (700, (300, 200)),
+             (1024, (1000, 999)), (600, (64, 3))]
     n_arr = np.array([c[0] for c in cases], dtype=np.int32)
     db = DeviceBatch(n_arr, seed=4)
     for i, (n, (r, c)) in enumerate(cases):

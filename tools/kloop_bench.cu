@@ -1,0 +1,138 @@
+// Microbenchmark (tool, not library): the left-looking panel-update k-loop in isolation —
+// TMA bulk copies into a full/empty mbarrier ring + DMMA m8n8k4 — to measure the DMMA rate
+// the pipeline sustains without the diagonal block / TRSM / stores. Each CTA repeatedly
+// computes acc(128 x NB) -= A[r0:r0+128, 0:K] * A[j0:j0+NB, 0:K]^T for row blocks of
+// synthetic column-major matrices (n = 1024, ldda = 1024) in HBM.
+// Variants: NB (32/64), KC, STAGES, warp tiling (8x1: 16 x NB per warp; 4x2: 32 x NB/2).
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o kloop_bench kloop_bench.cu
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e)); return 1; } } while (0)
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void dmma(double (&d)[2], double a, double b) {
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};" : "+d"(d[0]), "+d"(d[1]) : "d"(a), "d"(b));
+}
+__device__ __forceinline__ void mwait(uint64_t* b, uint32_t par) {
+  asm volatile("{\n .reg .pred p;\n W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}\n" :: "r"(su32(b)), "r"(par) : "memory");
+}
+
+template <int NB, int KC, int S, int WM, int WN>  // WM x WN warps, 8 warps total
+__global__ void __launch_bounds__(256, 2) kloop(const double* __restrict__ base, int nmat, int n, int K,
+                                                int blocks_per_cta, double* sink) {
+  constexpr int MB = 128, LDA = MB + 4, LDB = NB + 4;
+  constexpr int RW = MB / WM, CW = NB / WN, MT = RW / 8, NTT = CW / 8;
+  extern __shared__ __align__(128) unsigned char sm[];
+  double (*sa)[KC][LDA] = reinterpret_cast<double (*)[KC][LDA]>(sm);
+  double (*sb)[KC][LDB] = reinterpret_cast<double (*)[KC][LDB]>(sm + sizeof(double) * S * KC * LDA);
+  __shared__ uint64_t full[S], empty[S];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, g = lane >> 2, q = lane & 3;
+  const int wrow = (warp % WM) * RW, wcol = (warp / WM) * CW;
+  if (tid == 0) {
+    for (int i = 0; i < S; ++i) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(&full[i])));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(su32(&empty[i])));
+    }
+    asm volatile("fence.proxy.async.shared::cta;");
+  }
+  __syncthreads();
+  const int nk = K / KC;
+  const long total = (long)blocks_per_cta * nk;
+  auto chunk_src = [&](long c, int& kc, const double*& M, int& r0) {
+    const long blk = c / nk;
+    kc = (int)(c % nk);
+    const long gb = (long)blockIdx.x * blocks_per_cta + blk;
+    M = base + (size_t)(gb % nmat) * n * n;
+    r0 = K;  // rows below the panel
+  };
+  uint32_t prod = 0;
+  auto produce = [&]() {
+    if ((long)prod >= total) return;
+    int kc; const double* M; int r0;
+    chunk_src(prod, kc, M, r0);
+    const int st = prod % S; const uint32_t u = prod / S;
+    if (lane == 0) {
+      if (u > 0) mwait(&empty[st], (u - 1) & 1);
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(su32(&full[st])), "r"(KC * (MB + NB) * 8) : "memory");
+    }
+    __syncwarp();
+    if (lane < KC) {
+      const double* g0 = M + (size_t)(kc * KC + lane) * n + r0;
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                   :: "r"(su32(&sa[st][lane][0])), "l"(g0), "r"(MB * 8), "r"(su32(&full[st])) : "memory");
+    } else if (lane >= 16 && lane < 16 + KC) {
+      const double* g1 = M + (size_t)(kc * KC + lane - 16) * n + (K - NB);
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                   :: "r"(su32(&sb[st][lane - 16][0])), "l"(g1), "r"(NB * 8), "r"(su32(&full[st])) : "memory");
+    }
+    ++prod;
+  };
+  if (warp == 0) for (int i = 0; i < S - 1; ++i) produce();
+  double acc[MT][NTT][2] = {};
+  double keep = 0;
+  for (long c = 0; c < total; ++c) {
+    if (warp == 0) produce();
+    const int st = c % S;
+    mwait(&full[st], (c / S) & 1);
+#pragma unroll
+    for (int kk = 0; kk < KC / 4; ++kk) {
+      double fa[MT], fb[NTT];
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt) fa[mt] = -sa[st][kk * 4 + q][wrow + mt * 8 + g];
+#pragma unroll
+      for (int nt = 0; nt < NTT; ++nt) fb[nt] = sb[st][kk * 4 + q][wcol + nt * 8 + g];
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+    }
+    __syncwarp();
+    if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(su32(&empty[st])) : "memory");
+    if ((c + 1) % nk == 0) {  // end of a row block: fold acc (keeps the compiler honest)
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTT; ++nt) { keep += acc[mt][nt][0] + acc[mt][nt][1]; acc[mt][nt][0] = acc[mt][nt][1] = 0; }
+    }
+  }
+  if (keep == 1.2345) sink[0] = keep;
+}
+
+template <int NB, int KC, int S, int WM, int WN>
+int run(const double* base, int nmat, int n, int K, double* sink, int sms) {
+  constexpr int MB = 128;
+  size_t smem = sizeof(double) * S * KC * (MB + 4 + NB + 4);
+  CK(cudaFuncSetAttribute(kloop<NB, KC, S, WM, WN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ctas = 2 * sms, bpc = 24;
+  kloop<NB, KC, S, WM, WN><<<ctas, 256, smem>>>(base, nmat, n, K, 2, sink);
+  CK(cudaDeviceSynchronize());
+  cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+  cudaEventRecord(e0);
+  kloop<NB, KC, S, WM, WN><<<ctas, 256, smem>>>(base, nmat, n, K, bpc, sink);
+  cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
+  float ms; cudaEventElapsedTime(&ms, e0, e1);
+  double flops = 2.0 * ctas * bpc * (double)MB * NB * K;
+  printf("{\"NB\":%d,\"KC\":%d,\"S\":%d,\"warps\":\"%dx%d\",\"K\":%d,\"smem_KB\":%.1f,\"tflops\":%.2f}\n",
+         NB, KC, S, WM, WN, K, smem / 1024.0, flops / ms / 1e9);
+  return 0;
+}
+
+int main() {
+  const int n = 1024, nmat = 160;  // 1.34 GB of matrices (>> L2)
+  double* base; double* sink;
+  CK(cudaMalloc(&base, sizeof(double) * (size_t)nmat * n * n)); CK(cudaMalloc(&sink, 64));
+  CK(cudaMemset(base, 0, sizeof(double) * (size_t)nmat * n * n));
+  int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  for (int K : {256, 512}) {
+    run<64, 16, 3, 4, 2>(base, nmat, n, K, sink, sms);
+    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms);
+    run<64, 8, 5, 8, 1>(base, nmat, n, K, sink, sms);
+    run<64, 8, 5, 4, 2>(base, nmat, n, K, sink, sms);
+    run<64, 8, 8, 4, 2>(base, nmat, n, K, sink, sms);
+    run<32, 16, 3, 8, 1>(base, nmat, n, K, sink, sms);
+    run<64, 16, 4, 4, 2>(base, nmat, n, K, sink, sms);
+  }
+  return 0;
+}

@@ -1,0 +1,40 @@
+"""Phase breakdown of the v2 blocked kernel (debug build with -DVB_PHASE_PROF):
+python tools/phase_prof.py <lib.so> [config] [batch_limit]"""
+import ctypes
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+os.environ["VBATCHED_LIB"] = os.path.abspath(sys.argv[1])
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import vbgen  # noqa: E402
+import paper_conf_ipps_abdelfattahhtd16_b200 as vb  # noqa: E402
+from harness import DeviceBatch  # noqa: E402
+
+cfg = sys.argv[2] if len(sys.argv) > 2 else "C5"
+lim = int(sys.argv[3]) if len(sys.argv) > 3 else 0
+n = vbgen.sizes(cfg)
+if lim:
+    n = n[:lim]
+db = DeviceBatch(n, seed=vbgen.CONFIGS[cfg].seed).fill()
+L = vb.lib()
+L.vbatched_debug_phases.argtypes = [ctypes.c_void_p, ctypes.c_int]
+out = (ctypes.c_ulonglong * 8)()
+db.dpotrf()
+torch.cuda.synchronize()
+L.vbatched_debug_phases(ctypes.addressof(out), 1)
+db.fill()
+torch.cuda.synchronize()
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+db.dpotrf()
+e1.record()
+torch.cuda.synchronize()
+L.vbatched_debug_phases(ctypes.addressof(out), 1)
+names = ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "acc_init"]
+tot = out[4]
+print(f"{cfg} lim={lim} kernel {e0.elapsed_time(e1):.3f} ms; per-CTA-warp0 cycles (sum over CTAs):")
+for i, nm in enumerate(names):
+    print(f"  {nm:14s} {out[i]:16d}  {100.0 * out[i] / max(tot, 1):6.1f} %")
