@@ -167,11 +167,15 @@ int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owne
 }
 
 const char* vbatched_version(void) {
-  static char buf[256];
+  static char buf[320];
+  int occ[4] = {0, 0, 0, 0};
+  int dev_count = 0;
+  if (cudaGetDeviceCount(&dev_count) == cudaSuccess && dev_count > 0) potrf_occupancy(occ);
+  else cudaGetLastError();
   snprintf(buf, sizeof buf,
-           "libvbatched 0.2 (sm_100a; DMMA m8n8k4 f64; blocked NB=64 for n>%d, NB=32 for "
-           "32<n<=%d, MB=128; warp path n<=32)",
-           potrf_t64(), potrf_t64());
+           "libvbatched 0.3 (sm_100a; DMMA m8n8k4 f64; blocked NB=64 for n>%d, NB=32 for "
+           "32<n<=%d, MB=128; warp path n<=32; CTAs/SM v3=%d v2=%d v1=%d nb32=%d)",
+           potrf_t64(), potrf_t64(), occ[0], occ[1], occ[2], occ[3]);
   return buf;
 }
 

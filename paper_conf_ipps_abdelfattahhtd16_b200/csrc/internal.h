@@ -19,6 +19,7 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
                                cudaStream_t stream);
 
 int potrf_num_launches(int max_n_hint);
+void potrf_occupancy(int* out4);  // CTAs/SM of v3, v2, v1 NB64 and NB32 kernels
 
 // Stream-ordered scratch (pool-backed cudaMallocAsync).
 cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream);

@@ -697,13 +697,15 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
 // runs from registers and stores straight to global; the TMA stage ring is not aliased
 // with anything, so the producer (warp 0) keeps prefetching across the row blocks of a
 // panel; CTA-wide barriers only around the diagonal block and at the panel end.
-template <int NB_, int KC_, int STAGES_, int MINB_>
+template <int NB_, int KC_, int STAGES_, int MINB_, int WARPS_ = 8>
 struct Cfg2 {
   static constexpr int NB = NB_, KC = KC_, STAGES = STAGES_, MINB = MINB_;
-  static constexpr int WARPS = 8, THREADS = 256, MB = 128, NT = NB / 8;
+  static constexpr int WARPS = WARPS_;       // compute warps (16 rows each)
+  static constexpr int THREADS = 32 * WARPS, MB = 16 * WARPS, NT = NB / 8;
   static constexpr int LDA = MB + 4, LDB = NB + 4, LDT = NB + 4;
 };
 using Cfg64b = Cfg2<64, 16, 3, 2>;
+using Cfg64c = Cfg2<64, 16, 3, 2, 7>;  // v3: 7 compute warps + 1 producer warp = 256 threads
 
 template <class C>
 struct Smem2 {
@@ -718,6 +720,7 @@ struct Smem2 {
   double tv[C::NB];
   uint64_t full[C::STAGES];
   uint64_t empty[C::STAGES];
+  uint64_t panel_done;  // v3: one phase per panel (8 consumer-warp arrivals)
   uint32_t chunks;  // chunks issued so far (ring position)
   int item;
   int info;
@@ -726,9 +729,10 @@ struct Smem2 {
 // Diagonal 64x64 block by warps 0..3 (named barrier 1): L11 = potf2(C11), inv(L11) -> T12,
 // L21 = C21 inv(L11)^T -> T21, C22 -= L21 L21^T, L22 = potf2(C22), inv(L22) -> T11.
 // Stores L11, L21, L22 (rows < nb) to global (Ad, ld). Sets s.info (1-based, in-block).
-__device__ __noinline__ void diag_block64v2(Smem2<Cfg64b>& s, int nb, int wg, int lane,
-                                            double* Ad, int ld, bool below) {
-  constexpr int LDT = Cfg64b::LDT;
+template <class CC>
+__device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int lane, double* Ad,
+                                            int ld, bool below) {
+  constexpr int LDT = CC::LDT;
   double* T = &s.T[0][0];
   double* INV11 = T + 32 * LDT;  // T12 slot: INV11[k*LDT + n]
   double* INV22 = T;             // T11 slot (after L11 is dead)
@@ -824,8 +828,9 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, i
 
 // TRSM of this warp's 16 rows, in registers: X = C inv(L)^T (NB = 64: two 32-column steps
 // with inv(L11), L21, inv(L22) from s.T). Result overwrites acc.
-VB_DEVINL void trsm_regs64(Smem2<Cfg64b>& s, double (&acc)[2][8][2], int lane) {
-  constexpr int LDT = Cfg64b::LDT;
+template <class CC>
+VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
+  constexpr int LDT = CC::LDT;
   const double* T = &s.T[0][0];
   const int g = lane >> 2, q = lane & 3;
   double x[2][4][2];
@@ -1099,6 +1104,209 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
   }
 }
 
+// =======================================================================================
+// v3 blocked kernel (large n): v2 plus a dedicated TMA producer warp (warp 8). Measured in
+// tools/kloop_bench.cu: when a compute warp also produces, the k-loop stalls on the
+// producer/consumer handshake (16.6 TF/s at one CTA per SM); a producer warp that never
+// computes lifts it to 29 (one CTA) / 31.8 TF/s (two CTAs per SM). The producer walks the
+// same chunk sequence as the consumers; before the chunks of panel p it waits on the
+// panel_done mbarrier for panel p-1 (the consumers arrive after storing and fencing that
+// panel's L), so TMA never reads a column before it is final.
+constexpr int kV3Consumers = Cfg64c::WARPS;
+constexpr int kV3Threads = 32 * (kV3Consumers + 1);
+
+template <class C>
+VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int lane,
+                               uint32_t& gchunk, uint32_t& gpanel) {
+  constexpr int NB = C::NB, MB = C::MB, KC = C::KC;
+  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
+  const int npan = (n + NB - 1) / NB;
+  int done = npan;  // panels the consumers will complete for this matrix
+  fence_proxy_async();
+  for (int p = 1; p < npan; ++p) {
+    const int j0 = p * NB, nk = j0 / KC;
+    if (lane == 0) mbar_wait(&s.panel_done, (gpanel + p - 1) & 1);  // panel p-1 is stored
+    __syncwarp();
+    if (s.info) {  // the consumers failed in panel p-1 and stop there
+      done = p;
+      break;
+    }
+    for (int r0 = j0; r0 < n; r0 += MB) {
+      if (bulk && lane < min(NB, n - j0)) {  // warm L2 with this row block's panel values
+        const int rn = (min(MB, n - r0) + 1) & ~1;
+        bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * 8);
+      }
+      for (int kc = 0; kc < nk; ++kc) issue_chunk2<C>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
+    }
+  }
+  gpanel += done;
+}
+
+template <class C>
+VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int ld,
+                               int* info_out, uint32_t& gchunk, uint32_t& gpanel) {
+  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  const int wrow = warp * 16;
+  constexpr int CT = 32 * kV3Consumers;  // consumer threads (named barriers)
+  int npan_done = 0;
+  for (int j0 = 0; j0 < n; j0 += NB) {
+    const int nb = min(NB, n - j0);
+    const int nk = j0 / KC;
+    bool failed = false;
+    for (int r0 = j0; r0 < n; r0 += MB) {
+      const bool first = (r0 == j0);
+      const bool active = (r0 + wrow) < n;
+      if (failed) {  // drain this panel's remaining chunks (already issued by the producer)
+        for (int kc = 0; kc < nk; ++kc) {
+          const uint32_t gi = gchunk++;
+          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
+        }
+        continue;
+      }
+      double acc[2][NT][2];
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
+            const bool v = row < n && col < j0 + nb && row >= col;
+            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+          }
+      VB_T0(t_k)
+      for (int kc = 0; kc < nk; ++kc) {
+        const uint32_t gi = gchunk++;
+        const int st = gi % STAGES;
+        mbar_wait(&s.full[st], (gi / STAGES) & 1);
+        if (active) {
+#pragma unroll
+          for (int kk = 0; kk < KC / 4; ++kk) {
+            double fa[2], fb[NT];
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+              for (int nt = 0; nt < NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+          }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s.empty[st]);
+      }
+      VB_ADD(0, t_k)
+      VB_T0(t_d)
+      if (first) {
+        const bool below = r0 + nb < n;
+        const bool diag_warp = warp < NB / 16;
+        if (diag_warp) {
+#pragma unroll
+          for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+              s.T[nt * 8 + 2 * q][wrow + mt * 8 + g] = acc[mt][nt][0];
+              s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
+            }
+          bar_group(2, CT);
+          diag_block64v2(s, nb, warp, lane, A + (size_t)j0 * ld + j0, ld, below);
+          bar_group(3, CT);
+          failed = s.info != 0;
+        } else {
+          bar_group(2, CT);
+          bar_group(3, CT);
+          failed = s.info != 0;
+          if (!failed && below && active) {
+            trsm_regs64(s, acc, lane);
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+              for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                  const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
+                  if (row < n && row >= j0 + nb && col < nb)
+                    A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+                }
+          }
+        }
+        VB_ADD(1, t_d)
+        if (failed && tid == 0) *info_out = j0 + s.info;
+        continue;
+      }
+      VB_T0(t_t)
+      if (active) {
+        trsm_regs64(s, acc, lane);
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
+              if (row < n && col < nb) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+            }
+      }
+      VB_ADD(2, t_t)
+    }
+    // panel end: this warp's L stores are fenced for the async proxy, then released to the
+    // producer (which waits before issuing the next panel's reads of them)
+    fence_proxy_async_global();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&s.panel_done);
+    ++npan_done;
+    if (failed) break;
+  }
+  gpanel += npan_done;
+}
+
+__global__ void __launch_bounds__(kV3Threads, 2)
+    potrf_blocked3_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                          const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
+                          int range, int wait_upstream) {
+  using C = Cfg64c;
+  extern __shared__ __align__(128) unsigned char smem_raw3[];
+  Smem2<C>& s = *reinterpret_cast<Smem2<C>*>(smem_raw3);
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < C::STAGES; ++i) {
+      mbar_init(&s.full[i], 1);
+      mbar_init(&s.empty[i], kV3Consumers);
+    }
+    mbar_init(&s.panel_done, kV3Consumers);
+    s.info = 0;
+    fence_proxy_async();
+  }
+  __syncthreads();
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  uint32_t gchunk = 0, gpanel = 0;
+  for (;;) {
+    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
+    __syncthreads();
+    const int it = s.item;
+    __syncthreads();
+    if (it >= count) break;
+    const int m = order[start + it];
+    if (warp == kV3Consumers) {
+      produce_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
+    } else {
+      VB_T0(t_m)
+      consume_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gpanel);
+      VB_ADD(4, t_m)
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------------------
 constexpr int kWarpsPerCta = 2;
 struct WarpSmem {
@@ -1157,7 +1365,7 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 
 // ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
-static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0;
+static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0;
 static int g_t64 = -1;
 static int g_v2 = -1;
 
@@ -1199,9 +1407,16 @@ static cudaError_t init_device_info() {
                                                     Cfg64b::THREADS, sizeof(Smem2<Cfg64b>));
   if (e != cudaSuccess) return e;
   if (g_occ64b < 1) g_occ64b = 1;
+  e = cudaFuncSetAttribute(potrf_blocked3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)sizeof(Smem2<Cfg64c>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64c, potrf_blocked3_kernel, kV3Threads,
+                                                    sizeof(Smem2<Cfg64c>));
+  if (e != cudaSuccess) return e;
+  if (g_occ64c < 1) g_occ64c = 1;
   {
     const char* v = getenv("VB_V2");
-    g_v2 = v ? atoi(v) : 1;
+    g_v2 = v ? atoi(v) : 3;
   }
   potrf_t64();
   g_num_sms = sms;
@@ -1222,7 +1437,13 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.stream = stream;
   int wait = 1;  // the first factorisation kernel after the scan waits for it
   if (max_n_hint > g_t64) {
-    if (g_v2) {
+    if (g_v2 == 3) {
+      cfg.blockDim = dim3(kV3Threads);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64c)));
+      cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64c>);
+      e = cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 0,
+                             wait);
+    } else if (g_v2) {
       cfg.blockDim = dim3(Cfg64b::THREADS);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64b)));
       cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64b>);
@@ -1253,6 +1474,14 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
                                           g_num_sms * 8)));
   cfg.dynamicSmemBytes = 0;
   return cudaLaunchKernelEx(&cfg, potrf_warp_kernel, d_n, dA, d_ldda, d_info, ctrl, order, wait);
+}
+
+void potrf_occupancy(int* out4) {
+  init_device_info();
+  out4[0] = g_occ64c;
+  out4[1] = g_occ64b;
+  out4[2] = g_occ64;
+  out4[3] = g_occ32;
 }
 
 int potrf_num_launches(int max_n_hint) {

@@ -19,10 +19,10 @@ __device__ __forceinline__ void mwait(uint64_t* b, uint32_t par) {
   asm volatile("{\n .reg .pred p;\n W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}\n" :: "r"(su32(b)), "r"(par) : "memory");
 }
 
-template <int NB, int KC, int S, int WM, int WN>  // WM x WN warps, 8 warps total
-__global__ void __launch_bounds__(256, 2) kloop(const double* __restrict__ base, int nmat, int n, int K,
+template <int NB, int KC, int S, int WM, int WN, int MB = 128, int MINB = 2, int PRODW = 0>  // WM x WN warps (+1 producer)
+__global__ void __launch_bounds__(32 * (WM * WN + PRODW), MINB) kloop(const double* __restrict__ base, int nmat, int n, int K,
                                                 int blocks_per_cta, double* sink) {
-  constexpr int MB = 128, LDA = MB + 4, LDB = NB + 4;
+  constexpr int LDA = MB + 4, LDB = NB + 4, NW = WM * WN;
   constexpr int RW = MB / WM, CW = NB / WN, MT = RW / 8, NTT = CW / 8;
   extern __shared__ __align__(128) unsigned char sm[];
   double (*sa)[KC][LDA] = reinterpret_cast<double (*)[KC][LDA]>(sm);
@@ -33,7 +33,7 @@ __global__ void __launch_bounds__(256, 2) kloop(const double* __restrict__ base,
   if (tid == 0) {
     for (int i = 0; i < S; ++i) {
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(&full[i])));
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(su32(&empty[i])));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(su32(&empty[i])), "n"(NW));
     }
     asm volatile("fence.proxy.async.shared::cta;");
   }
@@ -69,11 +69,16 @@ __global__ void __launch_bounds__(256, 2) kloop(const double* __restrict__ base,
     }
     ++prod;
   };
-  if (warp == 0) for (int i = 0; i < S - 1; ++i) produce();
+  if (PRODW) {
+    if (warp == NW) {  // dedicated producer: run the whole ring, never compute
+      for (long c = 0; c < total; ++c) produce();
+      return;
+    }
+  } else if (warp == 0) for (int i = 0; i < S - 1; ++i) produce();
   double acc[MT][NTT][2] = {};
   double keep = 0;
   for (long c = 0; c < total; ++c) {
-    if (warp == 0) produce();
+    if (!PRODW && warp == 0) produce();
     const int st = c % S;
     mwait(&full[st], (c / S) & 1);
 #pragma unroll
@@ -100,22 +105,21 @@ __global__ void __launch_bounds__(256, 2) kloop(const double* __restrict__ base,
   if (keep == 1.2345) sink[0] = keep;
 }
 
-template <int NB, int KC, int S, int WM, int WN>
-int run(const double* base, int nmat, int n, int K, double* sink, int sms) {
-  constexpr int MB = 128;
+template <int NB, int KC, int S, int WM, int WN, int MB = 128, int MINB = 2, int PRODW = 0>
+int run(const double* base, int nmat, int n, int K, double* sink, int sms, int cps = 2) {
   size_t smem = sizeof(double) * S * KC * (MB + 4 + NB + 4);
-  CK(cudaFuncSetAttribute(kloop<NB, KC, S, WM, WN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int ctas = 2 * sms, bpc = 24;
-  kloop<NB, KC, S, WM, WN><<<ctas, 256, smem>>>(base, nmat, n, K, 2, sink);
+  CK(cudaFuncSetAttribute(kloop<NB, KC, S, WM, WN, MB, MINB, PRODW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ctas = cps * sms, bpc = 48 / cps;
+  kloop<NB, KC, S, WM, WN, MB, MINB, PRODW><<<ctas, 32 * (WM * WN + PRODW), smem>>>(base, nmat, n, K, 2, sink);
   CK(cudaDeviceSynchronize());
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   cudaEventRecord(e0);
-  kloop<NB, KC, S, WM, WN><<<ctas, 256, smem>>>(base, nmat, n, K, bpc, sink);
+  kloop<NB, KC, S, WM, WN, MB, MINB, PRODW><<<ctas, 32 * (WM * WN + PRODW), smem>>>(base, nmat, n, K, bpc, sink);
   cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
   float ms; cudaEventElapsedTime(&ms, e0, e1);
   double flops = 2.0 * ctas * bpc * (double)MB * NB * K;
-  printf("{\"NB\":%d,\"KC\":%d,\"S\":%d,\"warps\":\"%dx%d\",\"K\":%d,\"smem_KB\":%.1f,\"tflops\":%.2f}\n",
-         NB, KC, S, WM, WN, K, smem / 1024.0, flops / ms / 1e9);
+  printf("{\"NB\":%d,\"KC\":%d,\"S\":%d,\"warps\":\"%dx%d\",\"MB\":%d,\"K\":%d,\"cps\":%d,\"prodw\":%d,\"smem_KB\":%.1f,\"tflops\":%.2f}\n",
+         NB, KC, S, WM, WN, MB, K, cps, PRODW, smem / 1024.0, flops / ms / 1e9);
   return 0;
 }
 
@@ -125,14 +129,13 @@ int main() {
   CK(cudaMalloc(&base, sizeof(double) * (size_t)nmat * n * n)); CK(cudaMalloc(&sink, 64));
   CK(cudaMemset(base, 0, sizeof(double) * (size_t)nmat * n * n));
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-  for (int K : {256, 512}) {
-    run<64, 16, 3, 4, 2>(base, nmat, n, K, sink, sms);
-    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms);
-    run<64, 8, 5, 8, 1>(base, nmat, n, K, sink, sms);
-    run<64, 8, 5, 4, 2>(base, nmat, n, K, sink, sms);
-    run<64, 8, 8, 4, 2>(base, nmat, n, K, sink, sms);
-    run<32, 16, 3, 8, 1>(base, nmat, n, K, sink, sms);
-    run<64, 16, 4, 4, 2>(base, nmat, n, K, sink, sms);
+  for (int K : {256}) {
+    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms, 2);
+    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms, 1);
+    run<64, 16, 3, 8, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
+    run<64, 16, 4, 8, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
+    run<64, 16, 3, 8, 1, 128, 2, 1>(base, nmat, n, K, sink, sms, 2);
+    run<64, 16, 3, 16, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
   }
   return 0;
 }
