@@ -1125,18 +1125,28 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
   fence_proxy_async();
   for (int p = 1; p < npan; ++p) {
     const int j0 = p * NB, nk = j0 / KC;
+    // The first row block's chunks that read only columns < j0 - NB (final since before
+    // panel p-1 started) are issued before waiting for panel p-1: the ring does not drain
+    // at the panel boundary. Everything after them reads panel p-1's columns.
+    const int nk_free = (j0 - NB) / KC;
+    if (bulk && lane < min(NB, n - j0)) {
+      const int rn = (min(MB, n - j0) + 1) & ~1;
+      bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + j0, rn * 8);
+    }
+    for (int kc = 0; kc < nk_free; ++kc) issue_chunk2<C>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
     if (lane == 0) mbar_wait(&s.panel_done, (gpanel + p - 1) & 1);  // panel p-1 is stored
     __syncwarp();
-    if (s.info) {  // the consumers failed in panel p-1 and stop there
-      done = p;
+    if (s.info) {  // the consumers failed in panel p-1 and stop there (they also drain the
+      done = p;    // nk_free chunks issued above, see consume_matrix3)
       break;
     }
     for (int r0 = j0; r0 < n; r0 += MB) {
-      if (bulk && lane < min(NB, n - j0)) {  // warm L2 with this row block's panel values
+      if (r0 > j0 && bulk && lane < min(NB, n - j0)) {  // warm L2 with this block's panel values
         const int rn = (min(MB, n - r0) + 1) & ~1;
         bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * 8);
       }
-      for (int kc = 0; kc < nk; ++kc) issue_chunk2<C>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
+      for (int kc = (r0 == j0 ? nk_free : 0); kc < nk; ++kc)
+        issue_chunk2<C>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
     }
   }
   gpanel += done;
@@ -1260,7 +1270,19 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
     __syncwarp();
     if (lane == 0) mbar_arrive(&s.panel_done);
     ++npan_done;
-    if (failed) break;
+    if (failed) {
+      // the producer issued the next panel's first nk (= j0 / KC) independent chunks before
+      // it learnt of the failure: consume them too, so the ring stays consistent
+      if (j0 + NB < n) {
+        for (int kc = 0; kc < nk; ++kc) {
+          const uint32_t gi = gchunk++;
+          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
+        }
+      }
+      break;
+    }
   }
   gpanel += npan_done;
 }
