@@ -850,7 +850,8 @@ VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
 #pragma unroll
     for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
-      for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+      for (int nt = 0; nt < 4; ++nt)
+        if (4 * ks <= 8 * nt + 7) dmma(x[mt][nt], fa[mt], fb[nt]);  // inv(L11)^T is upper
   }
   // C2 -= X1 L21^T: B[k][n] = L21[n][k] = T[k][32 + n]
 #pragma unroll
@@ -886,7 +887,8 @@ VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
 #pragma unroll
     for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
-      for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
+      for (int nt = 0; nt < 4; ++nt)
+        if (4 * ks <= 8 * nt + 7) dmma(x[mt][nt], fa[mt], fb[nt]);  // inv(L22)^T is upper
   }
 #pragma unroll
   for (int mt = 0; mt < 2; ++mt)
@@ -1394,7 +1396,7 @@ static int g_v2 = -1;
 int potrf_t64() {
   if (g_t64 < 0) {
     const char* e = getenv("VB_T64");
-    g_t64 = e ? atoi(e) : 512;
+    g_t64 = e ? atoi(e) : 256;
     if (g_t64 < kWarpMaxN) g_t64 = kWarpMaxN;
   }
   return g_t64;

@@ -15,10 +15,16 @@ from harness import DeviceBatch  # noqa: E402
 
 cfg = sys.argv[2] if len(sys.argv) > 2 else "C5"
 lim = int(sys.argv[3]) if len(sys.argv) > 3 else 0
-n = vbgen.sizes(cfg)
+if cfg.startswith("u"):  # uniform size: u<n>x<count>
+    nn, cnt = (int(x) for x in cfg[1:].split("x"))
+    n = np.full(cnt, nn, dtype=np.int32)
+    seed = 3
+else:
+    n = vbgen.sizes(cfg)
+    seed = vbgen.CONFIGS[cfg].seed
 if lim:
     n = n[:lim]
-db = DeviceBatch(n, seed=vbgen.CONFIGS[cfg].seed).fill()
+db = DeviceBatch(n, seed=seed).fill()
 L = vb.lib()
 L.vbatched_debug_phases.argtypes = [ctypes.c_void_p, ctypes.c_int]
 out = (ctypes.c_ulonglong * 8)()
