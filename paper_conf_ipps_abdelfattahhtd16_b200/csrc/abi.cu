@@ -38,6 +38,8 @@ static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d
   if (batch < 0) return -6;
   if (check_max && max_n < 0) return -7;
   if (batch == 0) return 0;
+  if (check_max && max_n <= kWarpMaxN)  // all matrices on the warp path: no scan needed
+    return (int)launch_potrf_direct(d_n, dA, d_ldda, d_info, batch, max_n, stream);
   void* ws = nullptr;
   const size_t bytes = sizeof(Ctrl) + sizeof(int) * (size_t)batch;
   cudaError_t e = ws_alloc(&ws, bytes, stream);
@@ -83,6 +85,7 @@ int vbatched_dpotrf_scan(char uplo, const int* d_n, const int* d_ldda, int* d_in
   if (max_n < 0) return -6;
   if (batchCount == 0) return 0;
   if (!d_workspace) return -7;
+  if (max_n <= kWarpMaxN) return 0;  // the factor phase validates directly (no sort needed)
   Ctrl* ctrl = static_cast<Ctrl*>(d_workspace);
   return (int)launch_scan_bin(d_n, d_ldda, d_info, batchCount, max_n, true, ctrl,
                               reinterpret_cast<int*>(ctrl + 1), (cudaStream_t)stream);
@@ -94,8 +97,11 @@ int vbatched_dpotrf_factor(char uplo, const int* d_n, double* const* dA_array, c
   if (uplo != 'L' && uplo != 'l') return -1;
   if (batchCount < 0) return -6;
   if (max_n < 0) return -7;
-  if (batchCount == 0 || max_n == 0) return 0;
+  if (batchCount == 0) return 0;
   if (!d_workspace) return -8;
+  if (max_n <= kWarpMaxN)
+    return (int)launch_potrf_direct(d_n, dA_array, d_ldda, d_info, batchCount, max_n,
+                                    (cudaStream_t)stream);
   Ctrl* ctrl = static_cast<Ctrl*>(d_workspace);
   return (int)launch_potrf_paths(d_n, dA_array, d_ldda, d_info, batchCount, max_n, ctrl,
                                  reinterpret_cast<int*>(ctrl + 1), (cudaStream_t)stream);

@@ -1387,6 +1387,33 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
   }
 }
 
+// Direct warp path for batches whose max_n <= 32 (no scan, no sort: with every matrix this
+// small there is nothing to balance): warp w validates (info -2/-4/-7, as the scan would) and
+// factors matrices w, w + nwarps, ... One launch per call — the latency path for C1.
+__global__ void __launch_bounds__(32 * kWarpsPerCta)
+    potrf_warp_direct_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                             const int* __restrict__ d_ldda, int* __restrict__ d_info, int batch,
+                             int max_n) {
+  __shared__ WarpSmem s;
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  const int nw = gridDim.x * kWarpsPerCta;
+  for (int m = blockIdx.x * kWarpsPerCta + wi; m < batch; m += nw) {
+    const int n = d_n[m], ld = d_ldda[m];
+    int code = 0;
+    if (n < 0) code = -2;
+    else if (ld < (n > 1 ? n : 1)) code = -4;
+    else if (n > max_n) code = -7;
+    if (lane == 0) d_info[m] = code;
+    if (code != 0 || n == 0) continue;
+    if (n <= 8)
+      potrf_warp_matrix<8>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+    else if (n <= 16)
+      potrf_warp_matrix<16>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+    else
+      potrf_warp_matrix<32>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+  }
+}
+
 // ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
 static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0;
@@ -1510,7 +1537,18 @@ void potrf_occupancy(int* out4) {
 
 int potrf_num_launches(int max_n_hint) {
   init_device_info();
-  return 1 + (max_n_hint > kWarpMaxN ? 1 : 0) + (max_n_hint > g_t64 ? 1 : 0);
+  if (max_n_hint <= kWarpMaxN) return 1;  // direct warp kernel only
+  return 2 + 1 + (max_n_hint > potrf_t64() ? 1 : 0);
+}
+
+cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                                int batch, int max_n, cudaStream_t stream) {
+  cudaError_t e = init_device_info();
+  if (e != cudaSuccess) return e;
+  const int grid = std::max(1, std::min((batch + kWarpsPerCta - 1) / kWarpsPerCta, g_num_sms * 16));
+  potrf_warp_direct_kernel<<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info, batch,
+                                                                   max_n);
+  return cudaGetLastError();
 }
 
 }  // namespace vb

@@ -64,3 +64,4 @@ def test_host_api_argument_checks_and_codes():
 def test_kernel_launch_count():
     assert vb.vbatched_dpotrf_kernel_launches(0) == 0
     assert vb.vbatched_dpotrf_kernel_launches(32) == 1
+    assert vb.vbatched_dpotrf_kernel_launches(100) >= 3

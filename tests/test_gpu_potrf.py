@@ -267,6 +267,29 @@ def test_invalid_matrices_untouched():
     _check_batch(db, idxs=[0, 2])
 
 
+def test_direct_warp_path_validation():
+    """max_n <= 32 takes the scan-free direct warp kernel: it must validate like the scan
+    (-2 / -4 / -7, matrices untouched) and factor the rest."""
+    n = np.array([10, 30, 25, 3, 0, 31, 32], dtype=np.int32)
+    ld = np.array([32, 32, 32, 32, 1, 32, 32], dtype=np.int32)
+    db = DeviceBatch(n, ldda=ld, seed=6).fill(poison=True)
+    before = db.host_arena().copy()
+    bad_n = db.d_n.clone()
+    bad_n[3] = -1
+    bad_ld = db.d_ldda.clone()
+    bad_ld[1] = 29
+    from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
+    vbatched_dpotrf("L", bad_n, db.d_ptrs, bad_ld, db.d_info, db.B, 30)
+    torch.cuda.synchronize()
+    assert list(db.info()) == [0, -4, 0, -2, 0, -7, -7]
+    after = db.host_arena()
+    for i in (1, 3, 5, 6):
+        sl = slice(db.off[i], db.off[i] + int(ld[i]) * max(int(n[i]), 0))
+        assert np.array_equal(before[sl].view(np.uint64), after[sl].view(np.uint64))
+    _check_batch(db, idxs=[0, 2])
+    _check_sentinels(db, idxs=[0, 2])
+
+
 def test_argument_errors_and_empty():
     from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
     db = DeviceBatch(np.array([4], dtype=np.int32)).fill()
