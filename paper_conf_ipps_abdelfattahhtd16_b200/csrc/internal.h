@@ -8,6 +8,8 @@ namespace vb {
 
 // Size threshold above which matrices take the NB=64 blocked kernel (env VB_T64 overrides).
 int potrf_t64();
+// Size threshold up to which 32 < n matrices take the small-matrix kernel (env VB_TS).
+int potrf_ts();
 
 cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
                             bool check_max, Ctrl* ctrl, int* order, cudaStream_t stream);

@@ -318,6 +318,9 @@ VB_DEVINL void mm32_quarter(double (&acc)[2][2][2], int wg, int lane, FA fa, FB 
 VB_DEVINL void bar_group(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
 }
+VB_DEVINL void bar_group_arrive(int id, int nthreads) {
+  asm volatile("bar.arrive %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
+}
 
 // Diagonal block, NB = 64, by warps 0..3 (named barrier 1, 128 threads):
 //   L11 = potf2(C11); L21 = C21 inv(L11)^T; C22 -= L21 L21^T; L22 = potf2(C22).
@@ -1331,6 +1334,162 @@ __global__ void __launch_bounds__(kV3Threads, 2)
   }
 }
 
+// =======================================================================================
+// Small-matrix kernel (32 < n <= ts): one CTA of 2 warps per matrix, ~10 CTAs per SM, so
+// ~20 small matrices are in flight per SM (the regime is HBM/latency bound: C2). Left-
+// looking with NB = 32; within a panel the 32-row blocks alternate between the two warps
+// (block 0 = the diagonal block, always warp 0). Panel-update fragments are loaded straight
+// from L2 (__ldcg) into DMMA registers; the owning warp factors the diagonal block (POTF2 +
+// TRTRI in shared memory) and releases it to the other warp with a named barrier; TRSM runs
+// from registers and stores directly. One __syncthreads per panel.
+constexpr int kSmallWarps = 2;
+struct SmallSmem {
+  double T[32][36];    // diagonal block, T[c][r]
+  double inv[32][36];  // inv(L11) as TRSM B operand: inv[k][n] = X[n][k]
+  double S[16 * LDS_T];
+  double wbuf[64];
+  double sv[32];
+  double tv[32];
+  int item;
+  int info;
+};
+
+// acc (32 x 32 block at rows r0.., cols j0..) = A - L[r0:, 0:j0] L[j0:j0+32, 0:j0]^T
+VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restrict__ A, int n,
+                                  int ld, int r0, int j0, int nb, bool diag, int lane) {
+  const int g = lane >> 2, q = lane & 3;
+#pragma unroll
+  for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int row = r0 + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
+        const bool v = row < n && col < j0 + nb && (!diag || row >= col);
+        acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+      }
+  bool rv[4], cv[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    rv[t] = r0 + t * 8 + g < n;
+    cv[t] = j0 + t * 8 + g < n;
+  }
+#pragma unroll 2
+  for (int k = q; k < j0; k += 4) {
+    const double* col = A + (size_t)k * ld;
+    double fa[4], fb[4];
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      fa[t] = rv[t] ? -__ldcg(col + r0 + t * 8 + g) : 0.0;
+      fb[t] = cv[t] ? __ldcg(col + j0 + t * 8 + g) : 0.0;
+    }
+#pragma unroll
+    for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+  }
+}
+
+// X = C inv(L11)^T for a 32 x 32 block in registers (inv[k][n] upper in k,n: zero blocks
+// skipped), then direct stores of rows < n.
+VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], double* __restrict__ A,
+                                int n, int ld, int r0, int j0, int lane) {
+  const int g = lane >> 2, q = lane & 3;
+  double x[4][4][2];
+#pragma unroll
+  for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) x[mt][nt][0] = x[mt][nt][1] = 0.0;
+#pragma unroll
+  for (int ks = 0; ks < 8; ++ks) {
+    double fa[4], fb[4];
+#pragma unroll
+    for (int mt = 0; mt < 4; ++mt)
+      fa[mt] = cfrag_to_afrag(acc[mt][ks >> 1][0], acc[mt][ks >> 1][1], ks & 1, lane);
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt) fb[nt] = s.inv[ks * 4 + q][nt * 8 + g];
+#pragma unroll
+    for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt)
+        if (4 * ks <= 8 * nt + 7) dmma(x[mt][nt], fa[mt], fb[nt]);
+  }
+#pragma unroll
+  for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
+        if (row < n) A[(size_t)(j0 + col) * ld + row] = x[mt][nt][h];
+      }
+}
+
+__global__ void __launch_bounds__(32 * kSmallWarps, 8)
+    potrf_small_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                       const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                       const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
+                       int wait_upstream) {
+  __shared__ SmallSmem s;
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (;;) {
+    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
+    __syncthreads();
+    const int it = s.item;
+    __syncthreads();
+    if (it >= count) break;
+    const int m = order[start + it];
+    const int n = d_n[m], ld = d_ldda[m];
+    double* A = dA[m];
+    for (int j0 = 0; j0 < n; j0 += 32) {
+      const int nb = min(32, n - j0);
+      const int nblk = (n - j0 + 31) / 32;
+      bool failed = false;
+      for (int b = warp; b < nblk; b += kSmallWarps) {
+        const int r0 = j0 + 32 * b;
+        double acc[4][4][2];
+        small_panel_update(acc, A, n, ld, r0, j0, nb, b == 0, lane);
+        if (b == 0) {  // warp 0: the diagonal block
+          const int g = lane >> 2, q = lane & 3;
+#pragma unroll
+          for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt) {
+              s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+              s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+            }
+          __syncwarp();
+          const int info = potf2_block32(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
+                                         s.wbuf, s.sv, s.tv);
+          if (!info && nblk > 1)
+            trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
+          if (lane == 0) s.info = info;
+          failed = info != 0;
+          if (nblk > 1) bar_group_arrive(1, 32 * kSmallWarps);  // inv(L11) is ready
+        } else {
+          if (b == 1) {  // this warp's first block of the panel: wait for inv(L11)
+            bar_group(1, 32 * kSmallWarps);
+            failed = s.info != 0;
+          }
+          if (!failed) small_trsm_store(s, acc, A, n, ld, r0, j0, lane);
+        }
+        if (failed) break;
+      }
+      __syncthreads();  // the panel's L is stored (CTA scope) before the next panel reads it
+      if (s.info) {
+        if (tid == 0) d_info[m] = j0 + s.info;
+        break;
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // ---------------------------------------------------------------------------------------
 constexpr int kWarpsPerCta = 2;
 struct WarpSmem {
@@ -1368,12 +1527,12 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
   __shared__ WarpSmem s;
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
   if (wait_upstream) pdl_wait();
-  const int start = *(volatile const int*)&ctrl->start[2];
-  const int count = *(volatile const int*)&ctrl->count[2];
+  const int start = *(volatile const int*)&ctrl->start[3];
+  const int count = *(volatile const int*)&ctrl->count[3];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   for (;;) {
     int w = 0;
-    if (lane == 0) w = atomicAdd(&ctrl->head[2], 1);
+    if (lane == 0) w = atomicAdd(&ctrl->head[3], 1);
     w = __shfl_sync(kFull, w, 0);
     if (w >= count) break;
     const int m = order[start + w];
@@ -1418,7 +1577,18 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 static int g_num_sms = 0;
 static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0;
 static int g_t64 = -1;
+static int g_ts = -1;
+static int g_occ_small = 0;
 static int g_v2 = -1;
+
+int potrf_ts() {
+  if (g_ts < 0) {
+    const char* e = getenv("VB_TS");
+    g_ts = e ? atoi(e) : 128;
+    if (g_ts < kWarpMaxN) g_ts = kWarpMaxN;
+  }
+  return g_ts;
+}
 
 int potrf_t64() {
   if (g_t64 < 0) {
@@ -1469,6 +1639,11 @@ static cudaError_t init_device_info() {
     const char* v = getenv("VB_V2");
     g_v2 = v ? atoi(v) : 3;
   }
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_kernel,
+                                                    32 * kSmallWarps, 0);
+  if (e != cudaSuccess) return e;
+  if (g_occ_small < 1) g_occ_small = 1;
+  potrf_ts();
   potrf_t64();
   g_num_sms = sms;
   return cudaSuccess;
@@ -1510,12 +1685,21 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
     if (e != cudaSuccess) return e;
     wait = 0;
   }
-  if (max_n_hint > kWarpMaxN) {
+  if (max_n_hint > g_ts && g_ts < g_t64) {
     cfg.blockDim = dim3(Cfg32::THREADS);
     cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ32)));
     cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg32>);
     e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg32>, d_n, dA, d_ldda, d_info, ctrl, order,
                            1, wait);
+    if (e != cudaSuccess) return e;
+    wait = 0;
+  }
+  if (max_n_hint > kWarpMaxN) {
+    cfg.blockDim = dim3(32 * kSmallWarps);
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
+    cfg.dynamicSmemBytes = 0;
+    e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
+                           wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
@@ -1538,7 +1722,8 @@ void potrf_occupancy(int* out4) {
 int potrf_num_launches(int max_n_hint) {
   init_device_info();
   if (max_n_hint <= kWarpMaxN) return 1;  // direct warp kernel only
-  return 2 + 1 + (max_n_hint > potrf_t64() ? 1 : 0);
+  const int t64 = potrf_t64(), ts = potrf_ts();
+  return 3 + (max_n_hint > ts && ts < t64 ? 1 : 0) + (max_n_hint > t64 ? 1 : 0);
 }
 
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
