@@ -100,6 +100,18 @@ struct BlockedSmem {
 // Returns LAPACK info (1-based failing column; pivot !(d > 0) incl. NaN) or 0. On failure
 // columns < j hold L, the pivot d_j stays at (j,j) (lane j's a[j] == d_j), later entries are
 // partially updated. sv/tv (shared, >= NM doubles) receive l_cc and 1/l_cc.
+// 1/d for the LDL^T multipliers: hardware approximation + two Newton steps (within 1 ulp of
+// the IEEE quotient; exact for powers of two). Shorter than the IEEE division sequence on the
+// column-to-column chain. l_jj itself is still the IEEE correctly rounded sqrt.
+VB_DEVINL double rcp_nr(double d) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(d));
+  double e = fma(-d, r, 1.0);
+  r = fma(r, e, r);
+  e = fma(-d, r, 1.0);
+  return fma(r, e, r);
+}
+
 template <int NM>
 VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws, double* sv,
                               double* tv) {
@@ -115,7 +127,7 @@ VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws, dou
       break;
     }
     if (lane == j) myd = d;
-    const double rd = 1.0 / d;
+    const double rd = rcp_nr(d);
     const double u = a[j];
     const double w = u * rd;
     double* wb = ws + (j & 1) * 32;
@@ -263,22 +275,81 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
   __syncwarp();
 }
 
-// One warp: POTF2 of the nb x nb (nb <= 32) lower block at T (T[c*ldt + r]) in registers,
-// written back to T and to global (Ag, lda) — lower part, on failure up to the failing
-// column (incl. the pivot). Returns info.
+// One warp: POTF2 of the nb x nb (nb <= 32) lower block at T (T[c*ldt + r]), written back
+// to T and to global (Ag, lda) — lower part, on failure up to the failing column (incl. the
+// pivot). Blocked 16 + 16: POTF2 of columns 0..15 with all 32 rows in registers (which also
+// produces L21), the trailing 16x16 update C22 -= L21 L21^T on DMMA, POTF2 of C22.
+// sv/tv (>= 32 doubles) receive l_cc and 1/l_cc. Returns info.
 VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, int lda,
                             double* ws, double* sv, double* tv) {
-  double a[32];
+  const int nb1 = min(nb, 16), nb2 = nb - nb1;
+  int info;
+  {
+    double a[16];
 #pragma unroll
-  for (int c = 0; c < 32; ++c) a[c] = T[c * ldt + lane];
-  const int info = potf2_regs_warp<32>(a, nb, lane, ws, sv, tv);
-  const int ncol = info ? info : nb;
+    for (int c = 0; c < 16; ++c) a[c] = T[c * ldt + lane];
+    info = potf2_regs_warp<16>(a, nb1, lane, ws, sv, tv);
+    const int ncol = info ? info : nb1;
 #pragma unroll
-  for (int c = 0; c < 32; ++c)
-    if (c < ncol && lane >= c && lane < nb) {
-      T[c * ldt + lane] = a[c];
-      Ag[(size_t)c * lda + lane] = a[c];
+    for (int c = 0; c < 16; ++c)
+      if (c < ncol && lane >= c && lane < nb) {
+        T[c * ldt + lane] = a[c];
+        Ag[(size_t)c * lda + lane] = a[c];
+      }
+  }
+  __syncwarp();
+  if (info || nb2 <= 0) return info;
+  {  // C22 -= L21 L21^T (rows/cols 16..31; lower tiles only)
+    const int g = lane >> 2, q = lane & 3;
+    double acc[2][2][2];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          acc[mt][nt][h] = T[(16 + nt * 8 + 2 * q + h) * ldt + 16 + mt * 8 + g];
+#pragma unroll
+    for (int ks = 0; ks < 4; ++ks) {
+      double fa[2], fb[2];
+#pragma unroll
+      for (int t = 0; t < 2; ++t) {
+        fa[t] = -T[(ks * 4 + q) * ldt + 16 + t * 8 + g];
+        fb[t] = T[(ks * 4 + q) * ldt + 16 + t * 8 + g];
+      }
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 2; ++nt)
+          if (nt <= mt) dmma(acc[mt][nt], fa[mt], fb[nt]);
     }
+    __syncwarp();
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          if (nt <= mt) T[(16 + nt * 8 + 2 * q + h) * ldt + 16 + mt * 8 + g] = acc[mt][nt][h];
+  }
+  __syncwarp();
+  {  // POTF2 of C22: lanes 0..15 own its rows (lanes 16..31 mirror them, results unused)
+    const int r = lane & 15;
+    double* T22 = T + 16 * ldt + 16;
+    double a[16];
+#pragma unroll
+    for (int c = 0; c < 16; ++c) a[c] = T22[c * ldt + r];
+    const int info2 = potf2_regs_warp<16>(a, nb2, lane, ws, sv + 16, tv + 16);
+    const int ncol = info2 ? info2 : nb2;
+    double* A22 = Ag + (size_t)16 * lda + 16;
+#pragma unroll
+    for (int c = 0; c < 16; ++c)
+      if (lane < 16 && c < ncol && r >= c && r < nb2) {
+        T22[c * ldt + r] = a[c];
+        A22[(size_t)c * lda + r] = a[c];
+      }
+    info = info2 ? 16 + info2 : 0;
+  }
   __syncwarp();
   return info;
 }
@@ -1446,6 +1517,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     const int m = order[start + it];
     const int n = d_n[m], ld = d_ldda[m];
     double* A = dA[m];
+    VB_T0(t_m)
     for (int j0 = 0; j0 < n; j0 += 32) {
       const int nb = min(32, n - j0);
       const int nblk = (n - j0 + 31) / 32;
@@ -1453,7 +1525,9 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
       for (int b = warp; b < nblk; b += kSmallWarps) {
         const int r0 = j0 + 32 * b;
         double acc[4][4][2];
+        VB_T0(t_g)
         small_panel_update(acc, A, n, ld, r0, j0, nb, b == 0, lane);
+        VB_ADD(0, t_g)
         if (b == 0) {  // warp 0: the diagonal block
           const int g = lane >> 2, q = lane & 3;
 #pragma unroll
@@ -1464,10 +1538,14 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
               s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
             }
           __syncwarp();
+          VB_T0(t_p)
           const int info = potf2_block32(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
                                          s.wbuf, s.sv, s.tv);
+          VB_ADD(1, t_p)
+          VB_T0(t_i)
           if (!info && nblk > 1)
             trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
+          VB_ADD(2, t_i)
           if (lane == 0) s.info = info;
           failed = info != 0;
           if (nblk > 1) bar_group_arrive(1, 32 * kSmallWarps);  // inv(L11) is ready
@@ -1476,16 +1554,21 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
             bar_group(1, 32 * kSmallWarps);
             failed = s.info != 0;
           }
+          VB_T0(t_s)
           if (!failed) small_trsm_store(s, acc, A, n, ld, r0, j0, lane);
+          VB_ADD(3, t_s)
         }
         if (failed) break;
       }
+      VB_T0(t_b)
       __syncthreads();  // the panel's L is stored (CTA scope) before the next panel reads it
+      VB_ADD(5, t_b)
       if (s.info) {
         if (tid == 0) d_info[m] = j0 + s.info;
         break;
       }
     }
+    VB_ADD(4, t_m)
     __syncthreads();
   }
 }

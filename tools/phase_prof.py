@@ -39,7 +39,8 @@ db.dpotrf()
 e1.record()
 torch.cuda.synchronize()
 L.vbatched_debug_phases(ctypes.addressof(out), 1)
-names = ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "acc_init"]
+names = (["gemm", "potf2", "trtri", "trsm", "matrix_total", "panel_bar"] if os.environ.get("SMALL") else
+         ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "acc_init"])
 tot = out[4]
 print(f"{cfg} lim={lim} kernel {e0.elapsed_time(e1):.3f} ms; per-CTA-warp0 cycles (sum over CTAs):")
 for i, nm in enumerate(names):
