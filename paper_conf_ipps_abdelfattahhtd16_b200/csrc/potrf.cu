@@ -113,33 +113,36 @@ VB_DEVINL double rcp_nr(double d) {
 }
 
 template <int NM>
-VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws, double* sv,
+VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws_, double* sv,
                               double* tv) {
+  double* ws = static_cast<double*>(__builtin_assume_aligned(ws_, 16));
+  // Branch-free over the columns: the first failing pivot is recorded and the (garbage)
+  // work after it continues; only columns before it are scaled and stored, and lane j's
+  // a[j] (the failing pivot) is never modified after its column, so LAPACK's convention of
+  // leaving the pivot at (j,j) holds.
   int info = 0;
   double myd = 1.0;
   double dn = a[0];  // candidate next pivot (meaningful in lane j+1)
 #pragma unroll
   for (int j = 0; j < NM; ++j) {
-    if (j >= nb) break;
-    const double d = __shfl_sync(kFull, dn, j);
-    if (!(d > 0.0)) {
-      info = j + 1;
-      break;
-    }
-    if (lane == j) myd = d;
-    const double rd = rcp_nr(d);
-    const double u = a[j];
-    const double w = u * rd;
-    double* wb = ws + (j & 1) * 32;
-    wb[lane] = w;
-    if (j + 1 < NM) dn = fma(-u, w, a[(j + 1) < NM ? j + 1 : 0]);
-    __syncwarp();
+    if (j < nb) {
+      const double d = __shfl_sync(kFull, dn, j);
+      if (!(d > 0.0) && info == 0) info = j + 1;
+      if (lane == j) myd = d;
+      const double rd = rcp_nr(d);
+      const double u = a[j];
+      const double w = u * rd;
+      double* wb = ws + (j & 1) * 32;
+      wb[lane] = w;
+      if (j + 1 < NM) dn = fma(-u, w, a[(j + 1) < NM ? j + 1 : 0]);
+      __syncwarp();
 #pragma unroll
-    for (int k = j + 1; k < NM; ++k) a[k] = fma(-u, wb[k], a[k]);
+      for (int k = j + 1; k < NM; ++k) a[k] = fma(-u, wb[k], a[k]);
+    }
   }
   const int ncols = info ? info - 1 : nb;
   const double sq = sqrt(myd);
-  const double isq = 1.0 / sq;
+  const double isq = rcp_nr(sq);
   if (lane < ncols) {
     sv[lane] = sq;
     tv[lane] = isq;
@@ -1228,6 +1231,35 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
   gpanel += done;
 }
 
+// Consumer k-loop over nk chunks of the ring for this warp's 16 rows and the first NTL
+// 8-column tiles (NTL = 0: consume without computing — rows beyond n).
+template <class C, int NTL>
+VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk, int nk, int wrow,
+                       int lane) {
+  const int g = lane >> 2, q = lane & 3;
+  for (int kc = 0; kc < nk; ++kc) {
+    const uint32_t gi = gchunk++;
+    const int st = gi % C::STAGES;
+    mbar_wait(&s.full[st], (gi / C::STAGES) & 1);
+    if constexpr (NTL > 0) {
+#pragma unroll
+      for (int kk = 0; kk < C::KC / 4; ++kk) {
+        double fa[2], fb[NTL];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
+#pragma unroll
+        for (int nt = 0; nt < NTL; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NTL; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&s.empty[st]);
+  }
+}
+
 template <class C>
 VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int ld,
                                int* info_out, uint32_t& gchunk, uint32_t& gpanel) {
@@ -1265,26 +1297,19 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
             acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
           }
       VB_T0(t_k)
-      for (int kc = 0; kc < nk; ++kc) {
-        const uint32_t gi = gchunk++;
-        const int st = gi % STAGES;
-        mbar_wait(&s.full[st], (gi / STAGES) & 1);
-        if (active) {
-#pragma unroll
-          for (int kk = 0; kk < KC / 4; ++kk) {
-            double fa[2], fb[NT];
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
-#pragma unroll
-            for (int nt = 0; nt < NT; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-              for (int nt = 0; nt < NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
-          }
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&s.empty[st]);
+      // In a panel's first row block the diagonal-block warps only need the column tiles on
+      // or below their rows (SYRK): compile-time variants skip the strictly upper tiles.
+      const int ntl = (first && wrow < NB) ? (wrow + 16) / 8 : NT;
+      if (!active) {
+        k_loop3<C, 0>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 2) {
+        k_loop3<C, 2>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 4) {
+        k_loop3<C, 4>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 6) {
+        k_loop3<C, 6>(s, acc, gchunk, nk, wrow, lane);
+      } else {
+        k_loop3<C, NT>(s, acc, gchunk, nk, wrow, lane);
       }
       VB_ADD(0, t_k)
       VB_T0(t_d)
