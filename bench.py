@@ -398,7 +398,7 @@ def e2e_leg(args, cfg, db, n_loc, max_n, world, dev):
         return {"value": float(allv[:, 1].sum()) / tmax / 1e9, "unit": "GFLOP/s",
                 "h2d_bytes_per_step": payload + 16 * db.B, "d2h_bytes_per_step": payload + 4 * db.B,
                 "steps": args.e2e_steps, "s_per_step": tmax,
-                "api": "vbatched_dpotrf_host (pinned host buffers, 4 GiB device staging ring)"}
+                "api": "vbatched_dpotrf_host (pinned host buffers, 3-slot 6 GiB device staging ring)"}
     finally:
         vb.vbatched_host_free(hp)
 

@@ -97,7 +97,7 @@ int vbatched_dpotrf_factor(char uplo, const int* d_n, double* const* dA_array,
  * overlapping the factorisation. Each matrix's whole ldda x n column block is copied in
  * and back (the strict upper triangle and padding rows are returned unchanged).
  * Returns when every result is back in host memory. workspace_bytes bounds the device
- * staging memory (0 = library default, 4 GiB). Argument checks as vbatched_dpotrf
+ * staging memory (0 = library default, 6 GiB; the staging buffers are cached per device and reused by later calls). Argument checks as vbatched_dpotrf
  * (-2 n<0 and -4 ldda<max(1,n) are reported in h_info, -7 if n > max_n).
  * Extra return code: -9 = workspace_bytes too small for the largest matrix. */
 int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA_array, const int* h_ldda,

@@ -8,6 +8,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
+#include <mutex>
 #include <vector>
 
 #include "../../include/vbatched.h"
@@ -34,6 +35,7 @@ struct Chunk {
 struct Slot {
   cudaStream_t stream = nullptr;
   cudaEvent_t done = nullptr;
+  size_t dbuf_bytes = 0;
   char* dbuf = nullptr;     // matrices
   int* dmeta = nullptr;     // n[cap], ldda[cap], info[cap]
   double** dptr = nullptr;  // pointer array [cap]
@@ -42,6 +44,13 @@ struct Slot {
   int cap = 0;
   int chunk = -1;           // chunk whose results are in flight
 };
+
+struct StageCache {
+  Slot slots[kBufs];
+};
+constexpr int kMaxDevices = 64;
+StageCache g_stage[kMaxDevices];
+std::mutex g_stage_mutex;
 
 }  // namespace
 }  // namespace vb
@@ -55,7 +64,7 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
   if (batch < 0) return -6;
   if (max_n < 0) return -7;
   if (batch == 0) return 0;
-  if (workspace_bytes == 0) workspace_bytes = 4ull << 30;
+  if (workspace_bytes == 0) workspace_bytes = 6ull << 30;
   const size_t buf_bytes = (workspace_bytes / kBufs) & ~(size_t)255;
 
   // ---- host planning: validate (LAPACK codes), cut into chunks of <= buf_bytes
@@ -101,26 +110,45 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
   flush();
   if (chunks.empty()) return 0;
 
-  // ---- device/pinned resources
-  Slot slots[kBufs];
+  // ---- device/pinned resources: a per-process staging cache (grown on demand, reused by
+  // later calls on the same device; one caller at a time)
+  std::lock_guard<std::mutex> lock(g_stage_mutex);
   cudaError_t e = cudaSuccess;
+  int dev = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return (int)e;
+  Slot* slots = g_stage[dev].slots;
   const int nslots = std::min<int>(kBufs, (int)chunks.size());
+  size_t need = 0;
+  for (const Chunk& c : chunks) need = std::max(need, c.runs.back().dev_off + c.runs.back().bytes);
   cudaEvent_t start_ev = nullptr;
   e = cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventRecord(start_ev, (cudaStream_t)user_stream);
   for (int s = 0; s < nslots && e == cudaSuccess; ++s) {
     Slot& sl = slots[s];
-    sl.cap = max_cnt;
-    size_t need = 0;
-    for (const Chunk& c : chunks) need = std::max(need, c.runs.back().dev_off + c.runs.back().bytes);
-    if ((e = cudaStreamCreateWithFlags(&sl.stream, cudaStreamNonBlocking)) != cudaSuccess) break;
+    sl.chunk = -1;
+    if (!sl.stream && (e = cudaStreamCreateWithFlags(&sl.stream, cudaStreamNonBlocking)) != cudaSuccess) break;
     if ((e = cudaStreamWaitEvent(sl.stream, start_ev, 0)) != cudaSuccess) break;
-    if ((e = cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming)) != cudaSuccess) break;
-    if ((e = cudaMalloc(&sl.dbuf, need)) != cudaSuccess) break;
-    if ((e = cudaMalloc(&sl.dmeta, sizeof(int) * 3 * (size_t)sl.cap)) != cudaSuccess) break;
-    if ((e = cudaMalloc(&sl.dptr, sizeof(double*) * (size_t)sl.cap)) != cudaSuccess) break;
-    if ((e = cudaHostAlloc(&sl.hmeta, sizeof(int) * 3 * (size_t)sl.cap, 0)) != cudaSuccess) break;
-    if ((e = cudaHostAlloc(&sl.hptr, sizeof(double*) * (size_t)sl.cap, 0)) != cudaSuccess) break;
+    if (!sl.done && (e = cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming)) != cudaSuccess) break;
+    if (sl.dbuf_bytes < need) {
+      if (sl.dbuf) cudaFree(sl.dbuf);
+      sl.dbuf = nullptr;
+      sl.dbuf_bytes = 0;
+      if ((e = cudaMalloc(&sl.dbuf, need)) != cudaSuccess) break;
+      sl.dbuf_bytes = need;
+    }
+    if (sl.cap < max_cnt) {
+      if (sl.dmeta) cudaFree(sl.dmeta);
+      if (sl.dptr) cudaFree(sl.dptr);
+      if (sl.hmeta) cudaFreeHost(sl.hmeta);
+      if (sl.hptr) cudaFreeHost(sl.hptr);
+      sl.dmeta = nullptr; sl.dptr = nullptr; sl.hmeta = nullptr; sl.hptr = nullptr;
+      sl.cap = 0;
+      if ((e = cudaMalloc(&sl.dmeta, sizeof(int) * 3 * (size_t)max_cnt)) != cudaSuccess) break;
+      if ((e = cudaMalloc(&sl.dptr, sizeof(double*) * (size_t)max_cnt)) != cudaSuccess) break;
+      if ((e = cudaHostAlloc(&sl.hmeta, sizeof(int) * 3 * (size_t)max_cnt, 0)) != cudaSuccess) break;
+      if ((e = cudaHostAlloc(&sl.hptr, sizeof(double*) * (size_t)max_cnt, 0)) != cudaSuccess) break;
+      sl.cap = max_cnt;
+    }
   }
 
   auto drain = [&](Slot& sl) -> cudaError_t {  // wait for the slot's chunk, scatter info
@@ -170,17 +198,8 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
     cudaError_t r = drain(slots[s]);
     if (e == cudaSuccess) e = r;
   }
-  for (int s = 0; s < nslots; ++s) {
-    Slot& sl = slots[s];
-    if (sl.stream) cudaStreamSynchronize(sl.stream);
-    if (sl.dbuf) cudaFree(sl.dbuf);
-    if (sl.dmeta) cudaFree(sl.dmeta);
-    if (sl.dptr) cudaFree(sl.dptr);
-    if (sl.hmeta) cudaFreeHost(sl.hmeta);
-    if (sl.hptr) cudaFreeHost(sl.hptr);
-    if (sl.done) cudaEventDestroy(sl.done);
-    if (sl.stream) cudaStreamDestroy(sl.stream);
-  }
+  for (int s = 0; s < nslots; ++s)
+    if (slots[s].stream) cudaStreamSynchronize(slots[s].stream);
   if (start_ev) cudaEventDestroy(start_ev);
   return (int)e;
 }
