@@ -1598,6 +1598,147 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
   }
 }
 
+// =======================================================================================
+// Warp-per-matrix kernel for 32 < n <= ts (replaces the 2-warp small kernel by default):
+// one warp factors one matrix alone — no inter-warp synchronisation — and 16 single-warp
+// CTAs share an SM (~12 KB of shared memory each), so 16 small matrices are in flight per
+// SM. NB = 32 left-looking; 32-row blocks in sequence; panel-update fragments straight from
+// L2; POTF2 of the diagonal block in registers; the TRSM is a block substitution on DMMA
+// with the four 8x8 diagonal-block inverses of L11 (no full 32x32 inverse buffer):
+//   X_b = (C_b - sum_{c<b} X_c L_bc^T) inv(L_bb)^T,  b = 0..3 (8-column blocks).
+constexpr int LDW = 36;
+struct WSmem {
+  double T[32][LDW];       // diagonal block; L11 after POTF2
+  double inv8[4][8][9];    // inv(L_bb) as B operand: inv8[b][k][n] = inv(L_bb)[n][k]
+  double wbuf[64];
+  double sv[32];
+  double tv[32];
+};
+
+// Inverses of the four 8x8 diagonal blocks of L11 (T, tv = 1/l_cc): lane = (b, c) computes
+// column c of inv(L_bb) by substitution.
+VB_DEVINL void inv8_blocks(WSmem& s, int lane) {
+  const int b = lane >> 3, c = lane & 7, o = 8 * b;
+  double x[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    double acc = 0.0;
+#pragma unroll
+    for (int k = 0; k < i; ++k) acc = fma(s.T[o + k][o + i], x[k], acc);
+    const double r = s.tv[o + i];
+    x[i] = (i < c) ? 0.0 : ((i == c) ? r : -acc * r);
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) s.inv8[b][c][i] = x[i];  // [k=c][n=i] = inv[i][c]
+  __syncwarp();
+}
+
+// In-register TRSM of a 32 x 32 C block (C-fragment layout) against L11 by 8-column block
+// substitution; result stored to global rows < n.
+VB_DEVINL void wsmall_trsm_store(WSmem& s, double (&acc)[4][4][2], double* __restrict__ A, int n,
+                                 int ld, int r0, int j0, int lane) {
+  const int g = lane >> 2, q = lane & 3;
+#pragma unroll
+  for (int b = 0; b < 4; ++b) {
+    // C_b -= X_c L_bc^T for c < b:  B[k][n] = L[8b+n][8c+k] = T[8c+k][8b+n]
+#pragma unroll
+    for (int c = 0; c < b; ++c) {
+#pragma unroll
+      for (int ks = 0; ks < 2; ++ks) {
+        const double fb = s.T[8 * c + 4 * ks + q][8 * b + g];
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt) {
+          const double fa = -cfrag_to_afrag(acc[mt][c][0], acc[mt][c][1], ks, lane);
+          dmma(acc[mt][b], fa, fb);
+        }
+      }
+    }
+    // X_b = C_b inv(L_bb)^T
+    double x[4][2];
+#pragma unroll
+    for (int mt = 0; mt < 4; ++mt) x[mt][0] = x[mt][1] = 0.0;
+#pragma unroll
+    for (int ks = 0; ks < 2; ++ks) {
+      const double fb = s.inv8[b][4 * ks + q][g];
+#pragma unroll
+      for (int mt = 0; mt < 4; ++mt) {
+        const double fa = cfrag_to_afrag(acc[mt][b][0], acc[mt][b][1], ks, lane);
+        dmma(x[mt], fa, fb);
+      }
+    }
+#pragma unroll
+    for (int mt = 0; mt < 4; ++mt) {
+      acc[mt][b][0] = x[mt][0];
+      acc[mt][b][1] = x[mt][1];
+    }
+  }
+#pragma unroll
+  for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
+        if (row < n) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+      }
+}
+
+__global__ void __launch_bounds__(32, 16)
+    potrf_wsmall_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                        const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                        const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
+                        int wait_upstream) {
+  __shared__ __align__(16) WSmem s;
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int lane = threadIdx.x;
+  for (;;) {
+    int it = 0;
+    if (lane == 0) it = atomicAdd(&ctrl->head[range], 1);
+    it = __shfl_sync(kFull, it, 0);
+    if (it >= count) break;
+    const int m = order[start + it];
+    const int n = d_n[m], ld = d_ldda[m];
+    double* A = dA[m];
+    for (int j0 = 0; j0 < n; j0 += 32) {
+      const int nb = min(32, n - j0);
+      const int nblk = (n - j0 + 31) / 32;
+      int info = 0;
+      for (int b = 0; b < nblk; ++b) {
+        const int r0 = j0 + 32 * b;
+        double acc[4][4][2];
+        small_panel_update(acc, A, n, ld, r0, j0, nb, b == 0, lane);
+        if (b == 0) {
+          const int g = lane >> 2, q = lane & 3;
+#pragma unroll
+          for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt) {
+              s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+              s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+            }
+          __syncwarp();
+          info = potf2_block32(&s.T[0][0], LDW, nb, lane, A + (size_t)j0 * ld + j0, ld, s.wbuf,
+                               s.sv, s.tv);
+          if (info) break;
+          if (nblk > 1) inv8_blocks(s, lane);
+        } else {
+          wsmall_trsm_store(s, acc, A, n, ld, r0, j0, lane);
+        }
+      }
+      if (info) {
+        if (lane == 0) d_info[m] = j0 + info;
+        break;
+      }
+      // this warp stored the whole panel: its own later __ldcg reads see it (same thread order)
+      __syncwarp();
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------------------
 constexpr int kWarpsPerCta = 2;
 struct WarpSmem {
@@ -1686,7 +1827,8 @@ static int g_num_sms = 0;
 static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0;
 static int g_t64 = -1;
 static int g_ts = -1;
-static int g_occ_small = 0;
+static int g_occ_small = 0, g_occ_wsmall = 0;
+static int g_small = -1;
 static int g_v2 = -1;
 
 int potrf_ts() {
@@ -1751,6 +1893,13 @@ static cudaError_t init_device_info() {
                                                     32 * kSmallWarps, 0);
   if (e != cudaSuccess) return e;
   if (g_occ_small < 1) g_occ_small = 1;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_wsmall, potrf_wsmall_kernel, 32, 0);
+  if (e != cudaSuccess) return e;
+  if (g_occ_wsmall < 1) g_occ_wsmall = 1;
+  {
+    const char* v = getenv("VB_SMALL");
+    g_small = v ? atoi(v) : 2;
+  }
   potrf_ts();
   potrf_t64();
   g_num_sms = sms;
@@ -1803,11 +1952,19 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
     wait = 0;
   }
   if (max_n_hint > kWarpMaxN) {
-    cfg.blockDim = dim3(32 * kSmallWarps);
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
-    cfg.dynamicSmemBytes = 0;
-    e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
-                           wait);
+    if (g_small == 2) {
+      cfg.blockDim = dim3(32 * kSmallWarps);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
+      cfg.dynamicSmemBytes = 0;
+      e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
+                             wait);
+    } else {
+      cfg.blockDim = dim3(32);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
+      cfg.dynamicSmemBytes = 0;
+      e = cudaLaunchKernelEx(&cfg, potrf_wsmall_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
+                             wait);
+    }
     if (e != cudaSuccess) return e;
     wait = 0;
   }

@@ -153,6 +153,43 @@ print("OK")
     assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
 
 
+@pytest.mark.parametrize("small", ["1", "2"])
+def test_small_kernel_variants(small):
+    """Both small-matrix kernels (VB_SMALL=1 warp-per-matrix, 2 = two warps per matrix) on C2
+    sizes plus failing pivots in every 8-column sub-block (subprocess: the variant is read at
+    first use)."""
+    import subprocess
+    import sys
+    code = f"""
+import os, sys
+sys.path.insert(0, {repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))})
+import numpy as np, torch, vbgen
+from harness import DeviceBatch, compare_with_oracle
+n = np.concatenate([vbgen.sizes("C2")[:400], np.array([33, 40, 64, 65, 97, 128, 128, 100], np.int32)])
+fail = {{400: 1, 401: 9, 402: 17, 403: 40, 404: 70, 405: 128, 406: 100, 407: 33}}
+db = DeviceBatch(n, seed=12)
+inputs = {{}}
+for i in range(len(n)):
+    A = vbgen.f1_matrix(12, i, int(n[i]))
+    if i in fail:
+        k = fail[i]; A[k - 1, k - 1] = -A[k - 1, k - 1]
+    inputs[i] = A
+    db.set_matrix(i, A)
+db.dpotrf()
+torch.cuda.synchronize()
+info = db.info()
+for i in range(len(n)):
+    assert info[i] == fail.get(i, 0), (i, info[i])
+    r = compare_with_oracle(inputs[i], db.block(i), info[i])
+    assert r["ok"], (i, r)
+print("OK")
+"""
+    env = dict(os.environ, VB_SMALL=small)
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env,
+                         timeout=600)
+    assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
+
+
 def test_nan_info():
     cases = [(8, (2, 2)), (8, (5, 1)), (40, (33, 33)), (40, (39, 10)), (100, (70, 64)),
              (100, (0, 0)), (100, (99, 99)), (700, (40, 40)), (700, (300, 200)),
