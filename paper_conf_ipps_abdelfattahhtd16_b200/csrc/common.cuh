@@ -40,6 +40,15 @@ VB_DEVINL void dmma(double (&d)[2], double a, double b) {
       : "d"(a), "d"(b));
 }
 
+// p ? x : y through an opaque PTX selp, so that the compiler cannot rewrite a per-element
+// select over an unrolled register array into a dynamically indexed store.
+VB_DEVINL double selp(bool p, double x, double y) {
+  double r;
+  asm("{\n .reg .pred q;\n setp.ne.s32 q, %3, 0;\n selp.f64 %0, %1, %2, q;\n}\n"
+      : "=d"(r) : "d"(x), "d"(y), "r"((int)p));
+  return r;
+}
+
 VB_DEVINL uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }

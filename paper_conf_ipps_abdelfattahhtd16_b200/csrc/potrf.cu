@@ -48,6 +48,21 @@ __device__ unsigned long long g_phase[8];
 #define VB_T0(v)
 #define VB_ADD(i, v)
 #endif
+// Diagonal-block step timers (tools/diag_bench.cu built with -DVB_DIAG_PROF): thread 0
+// accumulates clock64() deltas between consecutive marks into g_dprof[i].
+#ifdef VB_DIAG_PROF
+__device__ unsigned long long g_dprof[16];
+#define DP_START long long dp_t = clock64();
+#define DP_MARK(i)                                                  \
+  if (threadIdx.x == 0) {                                           \
+    const long long dp_n = clock64();                               \
+    atomicAdd(&g_dprof[i], (unsigned long long)(dp_n - dp_t));      \
+    dp_t = dp_n;                                                    \
+  }
+#else
+#define DP_START
+#define DP_MARK(i)
+#endif
 
 template <int NB_, int MB_, int WARPS_M_, int WARPS_N_, int KC_, int STAGES_, int MINB_>
 struct BlockedCfg {
@@ -116,29 +131,29 @@ template <int NM>
 VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws_, double* sv,
                               double* tv) {
   double* ws = static_cast<double*>(__builtin_assume_aligned(ws_, 16));
-  // Branch-free over the columns: the first failing pivot is recorded and the (garbage)
-  // work after it continues; only columns before it are scaled and stored, and lane j's
-  // a[j] (the failing pivot) is never modified after its column, so LAPACK's convention of
-  // leaving the pivot at (j,j) holds.
+  // Branch-free over all NM columns: the caller pads rows/columns >= nb with the identity, so
+  // the padded pivots are 1 and leave the leading nb x nb factor untouched (no runtime branch
+  // around the shuffles, so a[] stays in registers). The first failing pivot (j < nb) is
+  // recorded and the (garbage) work after it continues; only columns before it are scaled
+  // and stored, and lane j's a[j] (the failing pivot) is never modified after its column, so
+  // LAPACK's convention of leaving the pivot at (j,j) holds.
   int info = 0;
   double myd = 1.0;
   double dn = a[0];  // candidate next pivot (meaningful in lane j+1)
 #pragma unroll
   for (int j = 0; j < NM; ++j) {
-    if (j < nb) {
-      const double d = __shfl_sync(kFull, dn, j);
-      if (!(d > 0.0) && info == 0) info = j + 1;
-      if (lane == j) myd = d;
-      const double rd = rcp_nr(d);
-      const double u = a[j];
-      const double w = u * rd;
-      double* wb = ws + (j & 1) * 32;
-      wb[lane] = w;
-      if (j + 1 < NM) dn = fma(-u, w, a[(j + 1) < NM ? j + 1 : 0]);
-      __syncwarp();
+    const double d = __shfl_sync(kFull, dn, j);
+    if (!(d > 0.0) && info == 0 && j < nb) info = j + 1;
+    if (lane == j) myd = d;
+    const double rd = rcp_nr(d);
+    const double u = a[j];
+    const double w = u * rd;
+    double* wb = ws + (j & 1) * 32;
+    wb[lane] = w;
+    if (j + 1 < NM) dn = fma(-u, w, a[(j + 1) < NM ? j + 1 : 0]);
+    __syncwarp();
 #pragma unroll
-      for (int k = j + 1; k < NM; ++k) a[k] = fma(-u, wb[k], a[k]);
-    }
+    for (int k = j + 1; k < NM; ++k) a[k] = fma(-u, wb[k], a[k]);
   }
   const int ncols = info ? info - 1 : nb;
   const double sq = sqrt(myd);
@@ -148,12 +163,13 @@ VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws_, do
     tv[lane] = isq;
   }
   __syncwarp();
+  // selects through opaque selp: written as `if (c == lane) a[c] = sq` the compiler turns the
+  // unrolled loop into one dynamically indexed store a[lane] = sq, which demotes a[] to local
+  // memory for the whole factorisation
 #pragma unroll
   for (int c = 0; c < NM; ++c) {
-    if (c < ncols) {
-      if (c < lane) a[c] *= tv[c];
-      else if (c == lane) a[c] = sq;
-    }
+    const double v = selp(c < lane, a[c] * tv[c], sq);
+    a[c] = selp(c < ncols && c <= lane, v, a[c]);
   }
   return info;
 }
@@ -288,9 +304,10 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
   const int nb1 = min(nb, 16), nb2 = nb - nb1;
   int info;
   {
-    double a[16];
+    double a[16];  // rows/columns outside the block: identity (potf2_regs_warp is branch-free)
 #pragma unroll
-    for (int c = 0; c < 16; ++c) a[c] = T[c * ldt + lane];
+    for (int c = 0; c < 16; ++c)
+      a[c] = (c < nb1 && lane < nb) ? T[c * ldt + lane] : selp(c == lane, 1.0, 0.0);
     info = potf2_regs_warp<16>(a, nb1, lane, ws, sv, tv);
     const int ncol = info ? info : nb1;
 #pragma unroll
@@ -341,7 +358,7 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
     double* T22 = T + 16 * ldt + 16;
     double a[16];
 #pragma unroll
-    for (int c = 0; c < 16; ++c) a[c] = T22[c * ldt + r];
+    for (int c = 0; c < 16; ++c) a[c] = (c < nb2 && r < nb2) ? T22[c * ldt + r] : selp(c == r, 1.0, 0.0);
     const int info2 = potf2_regs_warp<16>(a, nb2, lane, ws, sv + 16, tv + 16);
     const int ncol = info2 ? info2 : nb2;
     double* A22 = Ag + (size_t)16 * lda + 16;
@@ -816,12 +833,16 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
   const int g = lane >> 2, q = lane & 3;
   const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
   const int nb1 = min(nb, 32), nb2 = nb - nb1;
+  DP_START
   if (wg == 0) {
     const int info = potf2_block32(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
+    DP_MARK(0)
     if (!info && nb2 > 0) trtri32_dmma_warp(T, LDT, s.tv, INV11, LDT, s.S, LDS_T, lane);
+    DP_MARK(1)
     if (lane == 0) s.info = info;
   }
   bar_group(1, 128);
+  DP_MARK(2)
   if (s.info || nb2 == 0) return;
   {  // L21 = C21 inv(L11)^T
     double acc[2][2][2] = {};
@@ -840,6 +861,7 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
         }
   }
   bar_group(1, 128);
+  DP_MARK(3)
   {  // C22 -= L21 L21^T
     double acc[2][2][2];
 #pragma unroll
@@ -861,14 +883,18 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
           T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
   }
   bar_group(1, 128);
+  DP_MARK(4)
   if (wg == 0) {
     double* T22 = T + 32 * LDT + 32;
     const int info = potf2_block32(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf,
                                    s.sv + 32, s.tv + 32);
+    DP_MARK(5)
     if (!info && below) trtri32_dmma_warp(T22, LDT, s.tv + 32, INV22, LDT, s.S, LDS_T, lane);
+    DP_MARK(6)
     if (lane == 0) s.info = info ? 32 + info : 0;
   }
   bar_group(1, 128);
+  DP_MARK(7)
 }
 
 // Producer (warp 0): chunk kc of the row block at r0 into ring slot gi % STAGES.
@@ -1754,7 +1780,7 @@ VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* inf
   double a[NM];
 #pragma unroll
   for (int c = 0; c < NM; ++c)
-    a[c] = (c < n && lane >= c && lane < n) ? A[(size_t)c * ld + lane] : 0.0;
+    a[c] = (c < n && lane >= c && lane < n) ? A[(size_t)c * ld + lane] : selp(c == lane, 1.0, 0.0);
   const int info = potf2_regs_warp<NM>(a, n, lane, ws, sv, tv);
   const int ncol = info ? info : n;
 #pragma unroll

@@ -77,5 +77,18 @@ int main() {
              cudaGetErrorString(cudaGetLastError()));
     }
   }
+#ifdef VB_DIAG_PROF
+  {
+    cudaMemset(out, 0, 8);
+    unsigned long long z[16] = {};
+    cudaMemcpyToSymbol(g_dprof, z, sizeof z);
+    diag_kernel<<<148, 256, smem>>>(gA, 64, 50, out, 2);
+    cudaDeviceSynchronize();
+    unsigned long long h[16];
+    cudaMemcpyFromSymbol(h, g_dprof, sizeof h);
+    const char* st[8] = {"potf2_1", "trtri_1", "bar_1", "l21_mm_store", "syrk22", "potf2_2", "trtri_2", "bar_end"};
+    for (int i = 0; i < 8; ++i) printf("{\"diag64_step\":\"%s\",\"cycles\":%.0f}\n", st[i], h[i] / (148.0 * 50));
+  }
+#endif
   return 0;
 }
