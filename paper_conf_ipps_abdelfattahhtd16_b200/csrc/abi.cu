@@ -174,14 +174,15 @@ int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owne
 
 const char* vbatched_version(void) {
   static char buf[320];
-  int occ[4] = {0, 0, 0, 0};
+  int occ[4] = {0, 4, 0, 0};  // without a device: the default v3 width, occupancies unknown (0)
   int dev_count = 0;
   if (cudaGetDeviceCount(&dev_count) == cudaSuccess && dev_count > 0) potrf_occupancy(occ);
   else cudaGetLastError();
   snprintf(buf, sizeof buf,
-           "libvbatched 0.3 (sm_100a; DMMA m8n8k4 f64; blocked NB=64 for n>%d, NB=32 for "
-           "32<n<=%d, MB=128; warp path n<=32; CTAs/SM v3=%d v2=%d v1=%d nb32=%d)",
-           potrf_t64(), potrf_t64(), occ[0], occ[1], occ[2], occ[3]);
+           "libvbatched 0.4 (sm_100a; DMMA m8n8k4 f64; n>%d: NB=64 v3, %d compute warps + TMA "
+           "producer, %d CTAs/SM; %d<n<=%d: NB=32 8 warps, %d CTAs/SM; 32<n<=%d: small kernel, "
+           "%d CTAs/SM; n<=32: warp per matrix)",
+           potrf_t64(), occ[1], occ[0], potrf_ts(), potrf_t64(), occ[2], potrf_ts(), occ[3]);
   return buf;
 }
 

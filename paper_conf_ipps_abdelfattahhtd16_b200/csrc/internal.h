@@ -24,7 +24,7 @@ int potrf_num_launches(int max_n_hint);
 // max_n <= 32: one warp kernel that validates and factors directly (no scan).
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                 int batch, int max_n, cudaStream_t stream);
-void potrf_occupancy(int* out4);  // CTAs/SM of v3, v2, v1 NB64 and NB32 kernels
+void potrf_occupancy(int* out4);  // v3 CTAs/SM, v3 compute warps, NB32 CTAs/SM, small CTAs/SM
 
 // Stream-ordered scratch (pool-backed cudaMallocAsync).
 cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream);

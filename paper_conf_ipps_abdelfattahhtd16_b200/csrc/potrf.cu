@@ -681,6 +681,7 @@ VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, i
               issue_stage_bulk<C>(s, gi + STAGES - 1, kc + STAGES - 1, A, n, ld, r0, j0, lane);
             mbar_wait(&s.full[st], (gi / STAGES) & 1);
             if (warp_active) mma_chunk<C>(s, st, acc, wrow, wcol, g, q);
+            fence_proxy_async();  // this thread's LDS of the slot before the TMA refill (WAR)
             __syncwarp();
             if (lane == 0) mbar_arrive(&s.empty[st]);
           }
@@ -800,6 +801,7 @@ struct Cfg2 {
 };
 using Cfg64b = Cfg2<64, 16, 3, 2>;
 using Cfg64c = Cfg2<64, 16, 3, 2, 7>;  // v3: 7 compute warps + 1 producer warp = 256 threads
+using Cfg64d = Cfg2<64, 16, 2, 3, 4>;  // v3, 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer
 
 template <class C>
 struct Smem2 {
@@ -1079,6 +1081,7 @@ VB_DEVINL void potrf_blocked2_matrix(Smem2<C>& s, double* __restrict__ A, int n,
                 if (nt < ntl) dmma(acc[mt][nt], fa[mt], fb[nt]);
           }
         }
+        fence_proxy_async();  // this thread's LDS of the slot before the TMA refill (WAR)
         __syncwarp();
         if (lane == 0) mbar_arrive(&s.empty[st]);
       }
@@ -1217,8 +1220,6 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
 // same chunk sequence as the consumers; before the chunks of panel p it waits on the
 // panel_done mbarrier for panel p-1 (the consumers arrive after storing and fencing that
 // panel's L), so TMA never reads a column before it is final.
-constexpr int kV3Consumers = Cfg64c::WARPS;
-constexpr int kV3Threads = 32 * (kV3Consumers + 1);
 
 template <class C>
 VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int lane,
@@ -1280,6 +1281,11 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
 #pragma unroll
           for (int nt = 0; nt < NTL; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
       }
+      // Release of the slot to the TMA producer. The slot was read by generic-proxy LDS and is
+      // refilled through the async proxy: without this fence ptxas issues the arrive while the
+      // last LDS of the chunk are still in flight (their DMMAs are scheduled after it) and the
+      // refill can overtake them (a measured 1-in-10 run-to-run difference at C3).
+      fence_proxy_async();
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&s.empty[st]);
@@ -1293,7 +1299,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int g = lane >> 2, q = lane & 3;
   const int wrow = warp * 16;
-  constexpr int CT = 32 * kV3Consumers;  // consumer threads (named barriers)
+  constexpr int CT = 32 * C::WARPS;  // consumer threads (named barriers)
   int npan_done = 0;
   for (int j0 = 0; j0 < n; j0 += NB) {
     const int nb = min(NB, n - j0);
@@ -1414,12 +1420,13 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
   gpanel += npan_done;
 }
 
-__global__ void __launch_bounds__(kV3Threads, 2)
+template <class C>
+__global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     potrf_blocked3_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                           const int* __restrict__ d_ldda, int* __restrict__ d_info,
                           const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
                           int range, int wait_upstream) {
-  using C = Cfg64c;
+  constexpr int kV3Consumers = C::WARPS;
   extern __shared__ __align__(128) unsigned char smem_raw3[];
   Smem2<C>& s = *reinterpret_cast<Smem2<C>*>(smem_raw3);
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
@@ -1850,7 +1857,8 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 
 // ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
-static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0;
+static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0, g_occ64d = 0;
+static int g_v3w = 4;
 static int g_t64 = -1;
 static int g_ts = -1;
 static int g_occ_small = 0, g_occ_wsmall = 0;
@@ -1887,6 +1895,29 @@ static cudaError_t setup_kernel(int* occ) {
   return e;
 }
 
+template <class C>
+static cudaError_t setup_v3(int* occ) {
+  cudaError_t e = cudaFuncSetAttribute(potrf_blocked3_kernel<C>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)sizeof(Smem2<C>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked3_kernel<C>,
+                                                    32 * (C::WARPS + 1), sizeof(Smem2<C>));
+  if (*occ < 1) *occ = 1;
+  return e;
+}
+
+template <class C>
+static cudaError_t launch_v3(cudaLaunchConfig_t& cfg, int occ, int batch, const int* d_n,
+                             double* const* dA, const int* d_ldda, int* d_info, const Ctrl* ctrl,
+                             const int* order, int range, int wait) {
+  cfg.blockDim = dim3(32 * (C::WARPS + 1));
+  cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * occ)));
+  cfg.dynamicSmemBytes = sizeof(Smem2<C>);
+  return cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel<C>, d_n, dA, d_ldda, d_info, ctrl, order,
+                            range, wait);
+}
+
 static cudaError_t init_device_info() {
   if (g_num_sms) return cudaSuccess;
   int dev;
@@ -1904,13 +1935,12 @@ static cudaError_t init_device_info() {
                                                     Cfg64b::THREADS, sizeof(Smem2<Cfg64b>));
   if (e != cudaSuccess) return e;
   if (g_occ64b < 1) g_occ64b = 1;
-  e = cudaFuncSetAttribute(potrf_blocked3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)sizeof(Smem2<Cfg64c>));
-  if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64c, potrf_blocked3_kernel, kV3Threads,
-                                                    sizeof(Smem2<Cfg64c>));
-  if (e != cudaSuccess) return e;
-  if (g_occ64c < 1) g_occ64c = 1;
+  if ((e = setup_v3<Cfg64c>(&g_occ64c)) != cudaSuccess) return e;
+  if ((e = setup_v3<Cfg64d>(&g_occ64d)) != cudaSuccess) return e;
+  {
+    const char* v = getenv("VB_V3W");
+    g_v3w = v ? atoi(v) : 4;
+  }
   {
     const char* v = getenv("VB_V2");
     g_v2 = v ? atoi(v) : 3;
@@ -1947,11 +1977,10 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   int wait = 1;  // the first factorisation kernel after the scan waits for it
   if (max_n_hint > g_t64) {
     if (g_v2 == 3) {
-      cfg.blockDim = dim3(kV3Threads);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64c)));
-      cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64c>);
-      e = cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 0,
-                             wait);
+      if (g_v3w == 4)
+        e = launch_v3<Cfg64d>(cfg, g_occ64d, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
+      else
+        e = launch_v3<Cfg64c>(cfg, g_occ64c, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
     } else if (g_v2) {
       cfg.blockDim = dim3(Cfg64b::THREADS);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64b)));
@@ -2004,10 +2033,10 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
 
 void potrf_occupancy(int* out4) {
   init_device_info();
-  out4[0] = g_occ64c;
-  out4[1] = g_occ64b;
-  out4[2] = g_occ64;
-  out4[3] = g_occ32;
+  out4[0] = g_v3w == 4 ? g_occ64d : g_occ64c;
+  out4[1] = g_v3w == 4 ? Cfg64d::WARPS : Cfg64c::WARPS;
+  out4[2] = g_occ32;
+  out4[3] = g_small == 2 ? g_occ_small : g_occ_wsmall;
 }
 
 int potrf_num_launches(int max_n_hint) {

@@ -368,3 +368,26 @@ def test_host_api_chunked():
                          workspace_bytes=3 * 48 << 20)
     assert np.array_equal(info, dev.info())
     assert np.array_equal(host, dev.arena.cpu().numpy())
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C4"])
+def test_repeat_bit_identical(cfg):
+    """Every matrix is factored by one CTA in a fixed order, so repeated calls on the same input
+    must give bit-identical factors: any difference is a race (this caught a TMA-refill /
+    in-flight-LDS race in the ring that changed ~1 C3 run in 10)."""
+    c = vbgen.CONFIGS[cfg]
+    n = vbgen.sizes(c)
+    db = DeviceBatch(n, seed=c.seed, nonspd_mod=c.nonspd_mod)
+    ref = ref_info = None
+    scramble = torch.empty(1 << 27, dtype=torch.uint8, device="cuda")
+    for _ in range(15):
+        db.fill()
+        scramble.random_(0, 256)
+        db.dpotrf(max_n=c.nmax)
+        torch.cuda.synchronize()
+        out = db.arena.clone().view(torch.int64)
+        info = db.info()
+        if ref is None:
+            ref, ref_info = out, info
+            continue
+        assert torch.equal(out, ref) and np.array_equal(info, ref_info)
