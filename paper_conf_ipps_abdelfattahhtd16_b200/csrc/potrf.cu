@@ -64,6 +64,30 @@ __device__ unsigned long long g_dprof[16];
 #define DP_MARK(i)
 #endif
 
+// Optional per-matrix timeline (debug builds with -DVB_TIMELINE): the owning CTA/warp writes
+// (start ns, end ns, SM id, kernel) of each matrix to g_tl[4 m ..]; see tools/timeline.py.
+#ifdef VB_TIMELINE
+__device__ unsigned long long* g_tl;
+VB_DEVINL unsigned long long tl_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TL_BEGIN(v) const unsigned long long v = tl_now();
+#define TL_END(pred, v, m, kind)                               \
+  if ((pred) && g_tl) {                                        \
+    unsigned sm_;                                              \
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm_));           \
+    g_tl[4 * (size_t)(m)] = v;                                 \
+    g_tl[4 * (size_t)(m) + 1] = tl_now();                      \
+    g_tl[4 * (size_t)(m) + 2] = sm_;                           \
+    g_tl[4 * (size_t)(m) + 3] = kind;                          \
+  }
+#else
+#define TL_BEGIN(v)
+#define TL_END(pred, v, m, kind)
+#endif
+
 template <int NB_, int MB_, int WARPS_M_, int WARPS_N_, int KC_, int STAGES_, int MINB_>
 struct BlockedCfg {
   static constexpr int NB = NB_, MB = MB_, WARPS_M = WARPS_M_, WARPS_N = WARPS_N_;
@@ -782,8 +806,10 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
     __syncthreads();
     if (it >= count) break;
     const int m = order[start + it];
+    TL_BEGIN(t_tl)
     potrf_blocked_matrix<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m);
     __syncthreads();
+    TL_END(tid == 0, t_tl, m, 10 + range)
   }
 }
 
@@ -1453,6 +1479,7 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     __syncthreads();
     if (it >= count) break;
     const int m = order[start + it];
+    TL_BEGIN(t_tl)
     if (warp == kV3Consumers) {
       produce_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
     } else {
@@ -1460,6 +1487,7 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
       consume_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gpanel);
       VB_ADD(4, t_m)
     }
+    TL_END(tid == 0, t_tl, m, 30)
   }
 }
 
@@ -1576,6 +1604,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     const int n = d_n[m], ld = d_ldda[m];
     double* A = dA[m];
     VB_T0(t_m)
+    TL_BEGIN(t_tl)
     for (int j0 = 0; j0 < n; j0 += 32) {
       const int nb = min(32, n - j0);
       const int nblk = (n - j0 + 31) / 32;
@@ -1628,6 +1657,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     }
     VB_ADD(4, t_m)
     __syncthreads();
+    TL_END(tid == 0, t_tl, m, 20)
   }
 }
 
@@ -1819,12 +1849,14 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
     if (w >= count) break;
     const int m = order[start + w];
     const int n = d_n[m], ld = d_ldda[m];
+    TL_BEGIN(t_tl)
     if (n <= 8)
       potrf_warp_matrix<8>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else if (n <= 16)
       potrf_warp_matrix<16>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else
       potrf_warp_matrix<32>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+    TL_END(lane == 0, t_tl, m, 40)
   }
 }
 
@@ -2057,6 +2089,12 @@ cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_
 }
 
 }  // namespace vb
+
+#ifdef VB_TIMELINE
+extern "C" int vbatched_debug_timeline(unsigned long long* dptr) {
+  return (int)cudaMemcpyToSymbol(vb::g_tl, &dptr, sizeof(dptr));
+}
+#endif
 
 #ifdef VB_PHASE_PROF
 extern "C" int vbatched_debug_phases(unsigned long long* out, int reset) {
