@@ -1492,6 +1492,337 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
 }
 
 // =======================================================================================
+// v4 "team" kernel (large n): one CTA per SM = three independent matrix teams plus one diagonal
+// warp. Measured on B200 (tools/contention_bench.cu): a warp issuing back-to-back DMMAs starves
+// every other FP64 instruction (DFMA, DMUL and even dependent DMMAs) on the same SM sub-partition
+// — a 256-long DFMA chain takes 60x longer next to one DMMA-issuing warp and ~3700x next to two —
+// while FP32, integer and MUFU instructions are unaffected. In the v3 kernel the POTF2/TRTRI chain
+// of one CTA shares its sub-partitions with the other CTAs' k-loops, so the diagonal phase takes
+// 46 K cycles per 64x64 block under load instead of 21 K alone (25-30 % of a CTA's time for
+// n <= 512). Here the roles are pinned to sub-partitions (warp w runs on SMSP w % 4):
+//   SMSPs 0-2: 12 consumer warps, 4 per team (16 rows each of the team's 64-row blocks);
+//   SMSP 3:    one TMA producer warp per team (warps 3, 7, 11) and the diagonal warp (15),
+//              which factors every team's 64x64 diagonal blocks with no DMMA stream beside it.
+// The consumers hand the diagonal tile over (tile_ready mbarrier) and go straight on with the next
+// row block's panel update (look-ahead); they wait for the factor (diag_done) only before their
+// first TRSM of the panel.
+constexpr int kTeams = 3;
+constexpr int kTeamWarps = 16;
+
+struct TeamCtl {
+  uint64_t tile_ready;  // 4 consumer-warp arrivals per panel: the diagonal tile is in s.T
+  uint64_t diag_done;   // 1 arrival (diagonal warp): L11/L21/L22 stored, inverses in s.T, s.info
+  double* A;            // request: the matrix and its panel
+  int* info_out;
+  int ld, j0, nb, below;
+  int item;
+  volatile int done;  // the team has no more matrices
+};
+
+template <class C>
+struct alignas(128) TeamSlot {  // 128-byte aligned: the TMA destinations inside stay aligned
+  Smem2<C> s;
+};
+template <class C>
+struct TeamSmem {
+  TeamSlot<C> team[kTeams];
+  TeamCtl ctl[kTeams];
+};
+
+// Diagonal 64x64 block by ONE warp (same factorisation as diag_block64v2):
+//   L11 = potf2(C11), inv(L11) -> T12 slot; L21 = C21 inv(L11)^T -> T21 (and global);
+//   C22 -= L21 L21^T; L22 = potf2(C22), inv(L22) -> T11 slot. Sets s.info (in-block, 1-based).
+template <class CC>
+__device__ __noinline__ void diag_block64_1w(Smem2<CC>& s, int nb, int lane, double* Ad, int ld,
+                                             bool below) {
+  constexpr int LDT = CC::LDT;
+  double* T = &s.T[0][0];
+  double* INV11 = T + 32 * LDT;
+  double* INV22 = T;
+  const int g = lane >> 2, q = lane & 3;
+  const int nb1 = min(nb, 32), nb2 = nb - nb1;
+  int info = potf2_block32(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
+  if (info || nb2 <= 0) {
+    if (lane == 0) s.info = info;
+    __syncwarp();
+    return;
+  }
+  trtri32_dmma_warp(T, LDT, s.tv, INV11, LDT, s.S, LDS_T, lane);
+  {  // L21 = C21 inv(L11)^T: all four quarters in registers before T21 is overwritten
+    double acc[4][2][2][2];
+#pragma unroll
+    for (int wg = 0; wg < 4; ++wg)
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 2; ++nt) acc[wg][mt][nt][0] = acc[wg][mt][nt][1] = 0.0;
+#pragma unroll
+    for (int wg = 0; wg < 4; ++wg)
+      mm32_quarter(acc[wg], wg, lane, [&](int m, int k) { return T[k * LDT + 32 + m]; },
+                   [&](int k, int n) { return INV11[k * LDT + n]; });
+    __syncwarp();
+#pragma unroll
+    for (int wg = 0; wg < 4; ++wg) {
+      const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
+            T[c * LDT + r] = acc[wg][mt][nt][h];
+            if (r < nb) Ad[(size_t)c * ld + r] = acc[wg][mt][nt][h];
+          }
+    }
+  }
+  __syncwarp();
+  // C22 -= L21 L21^T on the three quarters on or below the diagonal (reads T21, writes T22)
+#pragma unroll
+  for (int wg = 0; wg < 4; ++wg) {
+    if (wg == 1) continue;
+    const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
+    double acc[2][2][2];
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          acc[mt][nt][h] = T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g];
+    mm32_quarter(acc, wg, lane, [&](int m, int k) { return -T[k * LDT + 32 + m]; },
+                 [&](int k, int n) { return T[k * LDT + 32 + n]; });
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
+  }
+  __syncwarp();
+  double* T22 = T + 32 * LDT + 32;
+  info = potf2_block32(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf, s.sv + 32,
+                       s.tv + 32);
+  if (!info && below) trtri32_dmma_warp(T22, LDT, s.tv + 32, INV22, LDT, s.S, LDS_T, lane);
+  if (lane == 0) s.info = info ? 32 + info : 0;
+  __syncwarp();
+}
+
+VB_DEVINL bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
+// Team consumer warp cw (0..3, rows 16cw..16cw+15 of each 64-row block) of one matrix.
+template <class C>
+VB_DEVINL void consume_matrix4(Smem2<C>& s, TeamCtl& x, double* __restrict__ A, int n, int ld,
+                               int* info_out, uint32_t& gchunk, uint32_t& gdiag, int cw, int lane,
+                               int cbar) {
+  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
+  static_assert(MB == NB, "the first row block of a panel is exactly its diagonal block");
+  const int g = lane >> 2, q = lane & 3;
+  const int wrow = cw * 16;
+  for (int j0 = 0; j0 < n; j0 += NB) {
+    const int nb = min(NB, n - j0);
+    const int nk = j0 / KC;
+    bool failed = false, waited = false;
+    for (int r0 = j0; r0 < n; r0 += MB) {
+      const bool first = (r0 == j0);
+      const bool active = (r0 + wrow) < n;
+      if (failed) {  // drain this panel's remaining chunks (already issued by the producer)
+        for (int kc = 0; kc < nk; ++kc) {
+          const uint32_t gi = gchunk++;
+          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
+        }
+        continue;
+      }
+      double acc[2][NT][2];
+#pragma unroll
+      for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
+            const bool v = row < n && col < j0 + nb && row >= col;
+            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+          }
+      const int ntl = first ? (wrow + 16) / 8 : NT;
+      if (!active) {
+        k_loop3<C, 0>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 2) {
+        k_loop3<C, 2>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 4) {
+        k_loop3<C, 4>(s, acc, gchunk, nk, wrow, lane);
+      } else if (ntl == 6) {
+        k_loop3<C, 6>(s, acc, gchunk, nk, wrow, lane);
+      } else {
+        k_loop3<C, NT>(s, acc, gchunk, nk, wrow, lane);
+      }
+      if (first) {  // hand the diagonal tile to the diagonal warp; go on with the next block
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt) {
+            s.T[nt * 8 + 2 * q][wrow + mt * 8 + g] = acc[mt][nt][0];
+            s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
+          }
+        if (cw == 0 && lane == 0) {
+          x.A = A;
+          x.info_out = info_out;
+          x.ld = ld;
+          x.j0 = j0;
+          x.nb = nb;
+          x.below = (j0 + nb < n) ? 1 : 0;
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&x.tile_ready);
+        continue;
+      }
+      if (!waited) {  // the first TRSM of the panel needs the diagonal factor
+        mbar_wait(&x.diag_done, gdiag & 1);
+        waited = true;
+        failed = s.info != 0;
+        if (failed) continue;
+      }
+      if (active) {
+        trsm_regs64(s, acc, lane);
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
+              if (row < n && col < nb) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+            }
+      }
+    }
+    if (!waited) {
+      mbar_wait(&x.diag_done, gdiag & 1);
+      failed = s.info != 0;
+    }
+    ++gdiag;
+    // panel end: this warp's L stores are fenced for the async proxy and released to the
+    // producer (the diagonal warp fenced the diagonal block's stores before diag_done)
+    fence_proxy_async_global();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&s.panel_done);
+    if (failed) {
+      if (j0 + NB < n) {  // the next panel's independent chunks the producer already issued
+        for (int kc = 0; kc < nk; ++kc) {
+          const uint32_t gi = gchunk++;
+          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
+        }
+      }
+      break;
+    }
+    bar_group(cbar, 128);  // every TRSM read of s.T is done before the next tile is written
+  }
+}
+
+template <class C>
+__global__ void __launch_bounds__(32 * kTeamWarps, 1)
+    potrf_team_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                      const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                      const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
+                      int wait_upstream) {
+  extern __shared__ __align__(128) unsigned char smem_raw4[];
+  TeamSmem<C>& S = *reinterpret_cast<TeamSmem<C>*>(smem_raw4);
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid < kTeams) {
+    Smem2<C>& s = S.team[tid].s;
+    for (int i = 0; i < C::STAGES; ++i) {
+      mbar_init(&s.full[i], 1);
+      mbar_init(&s.empty[i], 4);
+    }
+    mbar_init(&s.panel_done, 4);
+    s.info = 0;
+    mbar_init(&S.ctl[tid].tile_ready, 4);
+    mbar_init(&S.ctl[tid].diag_done, 1);
+    S.ctl[tid].done = 0;
+    fence_proxy_async();
+  }
+  __syncthreads();
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int sp = warp & 3;
+  if (warp == kTeamWarps - 1) {
+    // ---- diagonal warp: serve the teams' diagonal tiles as they become ready
+    uint32_t par[kTeams] = {0, 0, 0};
+    bool live[kTeams] = {true, true, true};
+    int nlive = kTeams;
+    while (nlive > 0) {
+      bool did = false;
+#pragma unroll
+      for (int t = 0; t < kTeams; ++t) {
+        if (!live[t]) continue;
+        TeamCtl& x = S.ctl[t];
+        if (mbar_test(&x.tile_ready, par[t])) {
+          par[t] ^= 1;
+          Smem2<C>& s = S.team[t].s;
+          double* Ad = x.A + (size_t)x.j0 * x.ld + x.j0;
+          diag_block64_1w(s, x.nb, lane, Ad, x.ld, x.below != 0);
+          if (s.info && lane == 0) *x.info_out = x.j0 + s.info;
+          fence_proxy_async_global();  // the diagonal block's L stores before later TMA reads
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&x.diag_done);
+          did = true;
+        } else if (x.done) {
+          live[t] = false;
+          --nlive;
+        }
+      }
+      if (!did) __nanosleep(32);
+    }
+    return;
+  }
+  int team, cw = -1;
+  if (sp == 3) {
+    team = warp >> 2;  // producers: warps 3, 7, 11
+  } else {
+    const int c = (warp >> 2) * 3 + sp;
+    team = c >> 2;
+    cw = c & 3;
+  }
+  Smem2<C>& s = S.team[team].s;
+  TeamCtl& x = S.ctl[team];
+  const int tbar = 1 + 2 * team, cbar = 2 + 2 * team;  // team (160 threads) / consumers (128)
+  uint32_t gchunk = 0, gpanel = 0, gdiag = 0;
+  for (;;) {
+    if (cw == 0 && lane == 0) x.item = atomicAdd(&ctrl->head[range], 1);
+    bar_group(tbar, 160);
+    const int it = x.item;
+    bar_group(tbar, 160);
+    if (it >= count) break;
+    const int m = order[start + it];
+    TL_BEGIN(t_tl)
+    if (cw < 0) {
+      produce_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
+    } else {
+      consume_matrix4<C>(s, x, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gdiag, cw, lane,
+                         cbar);
+    }
+    TL_END(cw == 0 && lane == 0, t_tl, m, 50)
+  }
+  if (cw == 0 && lane == 0) x.done = 1;
+}
+
+// =======================================================================================
 // Small-matrix kernel (32 < n <= ts): one CTA of 2 warps per matrix, ~10 CTAs per SM, so
 // ~20 small matrices are in flight per SM (the regime is HBM/latency bound: C2). Left-
 // looking with NB = 32; within a panel the 32-row blocks alternate between the two warps
@@ -1939,6 +2270,22 @@ static cudaError_t setup_v3(int* occ) {
   return e;
 }
 
+static int g_v4 = -1;
+static bool g_team_ok = false;
+
+template <class C>
+static cudaError_t setup_team() {
+  cudaError_t e = cudaFuncSetAttribute(potrf_team_kernel<C>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)sizeof(TeamSmem<C>));
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, potrf_team_kernel<C>, 32 * kTeamWarps,
+                                                    sizeof(TeamSmem<C>));
+  g_team_ok = (e == cudaSuccess && occ == 1);
+  return e;
+}
+
 template <class C>
 static cudaError_t launch_v3(cudaLaunchConfig_t& cfg, int occ, int batch, const int* d_n,
                              double* const* dA, const int* d_ldda, int* d_info, const Ctrl* ctrl,
@@ -1969,6 +2316,11 @@ static cudaError_t init_device_info() {
   if (g_occ64b < 1) g_occ64b = 1;
   if ((e = setup_v3<Cfg64c>(&g_occ64c)) != cudaSuccess) return e;
   if ((e = setup_v3<Cfg64d>(&g_occ64d)) != cudaSuccess) return e;
+  if ((e = setup_team<Cfg64d>()) != cudaSuccess) return e;
+  {
+    const char* v = getenv("VB_V4");
+    g_v4 = v ? atoi(v) : 0;
+  }
   {
     const char* v = getenv("VB_V3W");
     g_v3w = v ? atoi(v) : 4;
@@ -2009,10 +2361,17 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   int wait = 1;  // the first factorisation kernel after the scan waits for it
   if (max_n_hint > g_t64) {
     if (g_v2 == 3) {
-      if (g_v3w == 4)
+      if (g_v4 && g_team_ok) {
+        cfg.blockDim = dim3(32 * kTeamWarps);
+        cfg.gridDim = dim3(std::max(1, std::min((batch + kTeams - 1) / kTeams, g_num_sms)));
+        cfg.dynamicSmemBytes = sizeof(TeamSmem<Cfg64d>);
+        e = cudaLaunchKernelEx(&cfg, potrf_team_kernel<Cfg64d>, d_n, dA, d_ldda, d_info, ctrl,
+                               order, 0, wait);
+      } else if (g_v3w == 4) {
         e = launch_v3<Cfg64d>(cfg, g_occ64d, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
-      else
+      } else {
         e = launch_v3<Cfg64c>(cfg, g_occ64c, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
+      }
     } else if (g_v2) {
       cfg.blockDim = dim3(Cfg64b::THREADS);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64b)));
