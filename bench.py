@@ -322,7 +322,7 @@ def our_arm(args, cfg, rank, world, local_rank):
     roof["traffic"] = tr.get("bytes_per_launch") if tr else None
     if tr:
         roof["traffic_source"] = tr.get("source")
-    roof["kernel"] = "potrf_blocked_kernel<NB64|NB32> + potrf_warp_kernel (the factorisation launches)"
+    roof["kernel"] = "potrf_blocked3_kernel (NB=64) + potrf_small_kernel + potrf_warp_kernel (the factorisation launches)"
     roof["kernel_ms"] = sum(kern_ms) / args.steps
     roof["scan_ms"] = (sum(step_ms) - sum(kern_ms)) / args.steps
 

@@ -179,10 +179,9 @@ const char* vbatched_version(void) {
   if (cudaGetDeviceCount(&dev_count) == cudaSuccess && dev_count > 0) potrf_occupancy(occ);
   else cudaGetLastError();
   snprintf(buf, sizeof buf,
-           "libvbatched 0.4 (sm_100a; DMMA m8n8k4 f64; n>%d: NB=64 v3, %d compute warps + TMA "
-           "producer, %d CTAs/SM; %d<n<=%d: NB=32 8 warps, %d CTAs/SM; 32<n<=%d: small kernel, "
-           "%d CTAs/SM; n<=32: warp per matrix)",
-           potrf_t64(), occ[1], occ[0], potrf_ts(), potrf_t64(), occ[2], potrf_ts(), occ[3]);
+           "libvbatched 0.5 (sm_100a; DMMA m8n8k4 f64; n>%d: blocked NB=64, %d compute warps + TMA "
+           "producer, %d CTAs/SM; 32<n<=%d: small kernel, %d CTAs/SM; n<=32: warp per matrix)",
+           potrf_ts(), occ[1], occ[0], potrf_ts(), occ[3]);
   return buf;
 }
 

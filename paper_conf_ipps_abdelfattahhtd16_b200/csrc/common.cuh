@@ -14,19 +14,18 @@ namespace vb {
 constexpr unsigned kFull = 0xffffffffu;
 
 // Control block written by the scan (one per call, in the stream-ordered workspace).
-// The sorted work list order[] holds the valid matrices by n descending, split in four
+// The sorted work list order[] holds the valid matrices by n descending, split in three
 // contiguous ranges, one per factorisation kernel:
-//   range 0: n > t64          (blocked kernel, panel width 64)
-//   range 1: ts < n <= t64    (blocked kernel, panel width 32)
-//   range 2: 32 < n <= ts     (small-matrix kernel, 2 warps per matrix)
-//   range 3: 1 <= n <= 32     (warp-per-matrix kernel)
-constexpr int kRanges = 4;
+//   range 0: n > ts           (blocked kernel, panel width 64)
+//   range 1: 32 < n <= ts     (small-matrix kernel, 2 warps per matrix)
+//   range 2: 1 <= n <= 32     (warp-per-matrix kernel)
+constexpr int kRanges = 3;
 struct Ctrl {
   int head[kRanges];   // atomic queue heads (per range)
   int count[kRanges];  // matrices per range
   int start[kRanges];  // first position of each range in order[]
   int max_n;           // max n over valid matrices (for the _nomax interface / logging)
-  int pad[3];
+  int pad[6];
 };
 
 constexpr int kWarpMaxN = 32;  // warp-per-matrix path for n <= 32

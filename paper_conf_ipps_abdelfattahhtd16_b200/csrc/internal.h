@@ -6,9 +6,8 @@
 
 namespace vb {
 
-// Size threshold above which matrices take the NB=64 blocked kernel (env VB_T64 overrides).
-int potrf_t64();
-// Size threshold up to which 32 < n matrices take the small-matrix kernel (env VB_TS).
+// Size threshold: n > ts takes the NB=64 blocked kernel, 32 < n <= ts the small-matrix kernel
+// (env VB_TS, default 128).
 int potrf_ts();
 
 cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
@@ -24,7 +23,7 @@ int potrf_num_launches(int max_n_hint);
 // max_n <= 32: one warp kernel that validates and factors directly (no scan).
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                 int batch, int max_n, cudaStream_t stream);
-void potrf_occupancy(int* out4);  // v3 CTAs/SM, v3 compute warps, NB32 CTAs/SM, small CTAs/SM
+void potrf_occupancy(int* out4);  // blocked CTAs/SM, blocked compute warps, 0, small CTAs/SM
 
 // Stream-ordered scratch (pool-backed cudaMallocAsync).
 cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream);

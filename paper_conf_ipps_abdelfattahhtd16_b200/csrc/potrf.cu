@@ -3,25 +3,28 @@
 // Three persistent kernels drain the three ranges of the work list written by scan_bin
 // (matrices sorted by n descending = flops descending: longest-processing-time first):
 //
-//  * potrf_blocked_kernel<Cfg64>, n > t64, and potrf_blocked_kernel<Cfg32>, 32 < n <= t64:
-//    one CTA (8 warps) per matrix, the left-looking blocked Cholesky of PAPER.md Algorithm 1
-//     with panel width NB = 64 or 32:
-//      for each panel j0 (columns j0..j0+NB-1), for each block of MB = 128 rows r0 >= j0:
-//        panel update    C = A[r0:, j0:j0+NB] - L[r0:, 0:j0] L[j0:j0+NB, 0:j0]^T
+//  * potrf_blocked3_kernel, n > ts (128): one CTA (4 consumer warps + 1 TMA producer warp,
+//    3 CTAs per SM) per matrix, the left-looking blocked Cholesky of PAPER.md Algorithm 1
+//     with panel width NB = 64:
+//      for each panel j0 (columns j0..j0+63), for each block of MB = 64 rows r0 >= j0:
+//        panel update    C = A[r0:, j0:j0+64] - L[r0:, 0:j0] L[j0:j0+64, 0:j0]^T
 //                        ("customized syrk" with B a part of A, Fig. 2) on
-//                        the FP64 tensor cores (DMMA m8n8k4), operands staged by a cp.async
-//                        pipeline (double buffering); the accumulators start
-//                        from A's panel values, loaded before the k loop;
-//        tile factorize  L11 = chol(C1): POTF2 of 32-wide blocks by one warp, rows in
-//                        registers (LDL^T-form right-looking update so that sqrt and the
-//                        column scaling stay off the column-to-column chain); for NB = 64 the
-//                        64x64 block is done as POTF2(32) / TRSM / SYRK / POTF2(32);
-//        panel factorize C2 <- C2 L11^-T: TRTRI of L11 in shared memory (8x8 substitution +
-//                        recursive doubling on DMMA), then a DMMA GEMM — the trtri + gemm
-//                        TRSM design of PAPER.md:760-772.
-//    Every element of L is written once; earlier columns are re-read once per panel, so the
-//    HBM re-read traffic is ~ 8 n^3 / (6 NB) bytes per matrix: the wider panel is used
-//    where matrices are large enough to keep its longer diagonal chain amortised.
+//                        the FP64 tensor cores (DMMA m8n8k4), operands staged by TMA bulk
+//                        copies into an mbarrier ring fed by the producer warp (the paper's
+//                        double buffering); the accumulators start from A's
+//                        panel values;
+//        tile factorize  L11 = chol(C1) for the first row block (r0 == j0): the 64x64 block as
+//                        POTF2(32) / TRSM / SYRK / POTF2(32), each POTF2(32) = POTF2(16) in
+//                        registers (LDL^T-form right-looking update, short pivot chain) + DMMA
+//                        SYRK + POTF2(16);
+//        panel factorize C2 <- C2 L11^-T: TRTRI of the 32x32 diagonal blocks (8x8 substitution +
+//                        recursive doubling on DMMA), then DMMA against the triangular
+//                        inverses from registers — the trtri + gemm TRSM of PAPER.md:760-772.
+//    Every element of L is written once; earlier columns are re-read once per panel (HBM
+//    re-read traffic ~ 8 n^3 / (6 NB) bytes per matrix).
+//  * potrf_small_kernel, 32 < n <= ts: one 2-warp CTA per matrix, 8 CTAs per SM, NB = 32,
+//    panel-update fragments straight from L2 (potrf_wsmall_kernel, one warp per matrix, is the
+//    VB_SMALL=1 alternative).
 //  * potrf_warp_kernel, n <= 32: one warp per matrix, whole matrix in registers
 //    (the fused on-chip POTF2 of PAPER.md:551-560; one HBM read, one HBM write).
 // The kernels are chained with programmatic dependent launch: each releases its dependent
@@ -88,44 +91,7 @@ VB_DEVINL unsigned long long tl_now() {
 #define TL_END(pred, v, m, kind)
 #endif
 
-template <int NB_, int MB_, int WARPS_M_, int WARPS_N_, int KC_, int STAGES_, int MINB_>
-struct BlockedCfg {
-  static constexpr int NB = NB_, MB = MB_, WARPS_M = WARPS_M_, WARPS_N = WARPS_N_;
-  static constexpr int KC = KC_, STAGES = STAGES_, MINB = MINB_;
-  static constexpr int THREADS = 32 * WARPS_M * WARPS_N;
-  static constexpr int WM = MB / WARPS_M, WN = NB / WARPS_N;
-  static constexpr int MT = WM / 8, NT = WN / 8;
-  static constexpr int LDA = MB + 4;  // padded smem leading dims: conflict-free fragments
-  static constexpr int LDB = NB + 4;
-  static constexpr int LDI = NB + 4;
-};
-using Cfg32 = BlockedCfg<32, 128, 8, 1, 16, 3, 3>;
-using Cfg64 = BlockedCfg<64, 128, 4, 2, 16, 3, 2>;
-
 constexpr int LDS_T = 18;  // TRTRI32 scratch leading dim (16 columns used)
-
-template <class C>
-struct BlockedSmem {
-  union {
-    struct {
-      double a[C::STAGES][C::KC][C::LDA];  // A chunk: [k][row]
-      double b[C::STAGES][C::KC][C::LDB];  // B chunk: [k][panel row]
-    } pipe;
-    struct {
-      double tile[C::NB][C::LDA];  // C tile: [col][row], aliases the pipeline after the k loop
-      double scratch[16 * LDS_T];  // TRTRI32 scratch
-      double wbuf[64];
-      double sv[C::NB];
-      double tv[C::NB];
-    } e;
-  } u;
-  double inv[C::NB][C::LDI];  // inv[k][n] = (L11^-1)[n][k]  (DMMA B operand of the TRSM)
-  uint64_t full[C::STAGES];   // TMA ring: stage filled (producer arrive.expect_tx + bytes)
-  uint64_t empty[C::STAGES];  // TMA ring: stage consumed (one arrive per warp)
-  uint32_t chunks;            // chunks issued so far by this CTA (ring position)
-  int item;
-  int info;
-};
 
 // ---------------------------------------------------------------------------------------
 // POTF2 of an nb x nb (nb <= NM <= 32) lower block by one warp, lane r holding row r in
@@ -398,18 +364,6 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
   return info;
 }
 
-// Diagonal block, NB = 32 (warp 0 only). Sets s.info; builds s.inv when rows follow below.
-// Out of line so that its register footprint does not spill into the caller's k-loop.
-__device__ __noinline__ void diag_block32(BlockedSmem<Cfg32>& s, int nb, int lane, double* Ad,
-                                          int ld, bool below) {
-  const int info = potf2_block32(&s.u.e.tile[0][0], Cfg32::LDA, nb, lane, Ad, ld, s.u.e.wbuf,
-                                 s.u.e.sv, s.u.e.tv);
-  if (!info && below)
-    trtri32_dmma_warp(&s.u.e.tile[0][0], Cfg32::LDA, s.u.e.tv, &s.inv[0][0], Cfg32::LDI,
-                      s.u.e.scratch, LDS_T, lane);
-  if (lane == 0) s.info = info;
-}
-
 // 32x32x32 DMMA products on a 4-warp group (wg = warp index 0..3): each warp owns a 16x16
 // quarter (2x2 tiles). acc[m][n] += sum_k fa(m,k) fb(k,n) over k = 0..31.
 template <class FA, class FB>
@@ -437,387 +391,10 @@ VB_DEVINL void bar_group_arrive(int id, int nthreads) {
   asm volatile("bar.arrive %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// Diagonal block, NB = 64, by warps 0..3 (named barrier 1, 128 threads):
-//   L11 = potf2(C11); L21 = C21 inv(L11)^T; C22 -= L21 L21^T; L22 = potf2(C22).
-// For the TRSM of the rows below (two 32-column steps, 32x32 inverses only, as PAPER.md:
-// 762-766 prescribes) it leaves in s.inv: inv(L11) in [0:32][0:32], L21^T in [0:32][32:64]
-// (inv[k][32+n] = L21[n][k]) and inv(L22) in [32:64][32:64], all as B operands
-// (inv[k][n] = X[n][k]). T = the C tile (T[c*LDA + r]). Sets s.info (1-based, in-block).
-__device__ __noinline__ void diag_block64(BlockedSmem<Cfg64>& s, int nb, int wg, int lane,
-                                          double* Ad, int ld, bool below) {
-  constexpr int LDA = Cfg64::LDA, LDI = Cfg64::LDI;
-  double* T = &s.u.e.tile[0][0];
-  double* INV = &s.inv[0][0];
-  const int g = lane >> 2, q = lane & 3;
-  const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
-  const int nb1 = min(nb, 32), nb2 = nb - nb1;
-  // (1) L11 = potf2(C11) and inv(L11) (warp 0); TRTRI scratch in INV[32:48][0:20] (unused)
-  if (wg == 0) {
-    const int info = potf2_block32(T, LDA, nb1, lane, Ad, ld, s.u.e.wbuf, s.u.e.sv, s.u.e.tv);
-    if (!info && nb2 > 0) trtri32_dmma_warp(T, LDA, s.u.e.tv, INV, LDI, INV + 32 * LDI, LDI, lane);
-    if (lane == 0) s.info = info;
-  }
-  bar_group(1, 128);
-  if (s.info || nb2 == 0) return;
-  // (2) L21 = C21 inv(L11)^T  (C21 = T rows 32..63, cols 0..31); B[k][n] = X11[n][k] = INV[k][n]
-  {
-    double acc[2][2][2] = {};
-    mm32_quarter(acc, wg, lane, [&](int m, int k) { return T[k * LDA + 32 + m]; },
-                 [&](int k, int n) { return INV[k * LDI + n]; });
-    bar_group(1, 128);  // all reads of C21 done
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
-          T[c * LDA + r] = acc[mt][nt][h];
-          INV[c * LDI + r] = acc[mt][nt][h];  // L21^T: inv[k=c][32+n] with n = r-32
-          if (r < nb) Ad[(size_t)c * ld + r] = acc[mt][nt][h];
-        }
-  }
-  bar_group(1, 128);
-  // (3) C22 -= L21 L21^T (T rows/cols 32..63)
-  {
-    double acc[2][2][2];
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          acc[mt][nt][h] = T[(32 + n0 + nt * 8 + 2 * q + h) * LDA + 32 + m0 + mt * 8 + g];
-    mm32_quarter(acc, wg, lane, [&](int m, int k) { return -T[k * LDA + 32 + m]; },
-                 [&](int k, int n) { return T[k * LDA + 32 + n]; });
-    bar_group(1, 128);
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          T[(32 + n0 + nt * 8 + 2 * q + h) * LDA + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
-  }
-  bar_group(1, 128);
-  // (4) L22 = potf2(C22) and inv(L22) (warp 0); TRTRI scratch in INV[32:48][0:20] (unused)
-  if (wg == 0) {
-    double* T22 = T + 32 * LDA + 32;
-    const int info = potf2_block32(T22, LDA, nb2, lane, Ad + (size_t)32 * ld + 32, ld,
-                                   s.u.e.wbuf, s.u.e.sv + 32, s.u.e.tv + 32);
-    if (!info && below)
-      trtri32_dmma_warp(T22, LDA, s.u.e.tv + 32, INV + 32 * LDI + 32, LDI, INV + 32 * LDI, LDI,
-                        lane);
-    if (lane == 0) s.info = info ? 32 + info : 0;
-  }
-  bar_group(1, 128);
-}
-
-// Stage k-chunk kc of the panel-update operands: A rows r0..r0+MB-1 and the panel rows
-// j0..j0+NB-1 (the "B" of Fig. 2), columns kc*KC..kc*KC+KC-1. Rows >= n are zero-filled.
-template <class C>
-VB_DEVINL void load_stage(BlockedSmem<C>& s, int st, int kc, const double* __restrict__ A, int n,
-                          int ld, int r0, int j0) {
-  const int tid = threadIdx.x;
-  const int k0 = kc * C::KC;
-#pragma unroll
-  for (int e = 0; e < (C::MB * C::KC) / C::THREADS; ++e) {
-    const int idx = tid + e * C::THREADS;
-    const int c = idx / C::MB, r = idx % C::MB;
-    const int row = r0 + r;
-    const bool p = row < n;
-    cp_async8(&s.u.pipe.a[st][c][r], A + (p ? (size_t)(k0 + c) * ld + row : 0), p);
-  }
-#pragma unroll
-  for (int e = 0; e < (C::NB * C::KC) / C::THREADS; ++e) {
-    const int idx = tid + e * C::THREADS;
-    const int c = idx / C::NB, r = idx % C::NB;
-    const int row = j0 + r;
-    const bool p = row < n;
-    cp_async8(&s.u.pipe.b[st][c][r], A + (p ? (size_t)(k0 + c) * ld + row : 0), p);
-  }
-}
-
-// TRSM of the 128 x NB C tile by its warps (warp w owns rows 16w..16w+15), in place.
-// B operands from s.inv (see diag_block64 / trtri32_dmma_warp for the layout).
-template <class C>
-VB_DEVINL void trsm_rows16(BlockedSmem<C>& s, int warp, int lane, bool active) {
-  const int g = lane >> 2, q = lane & 3;
-  const int r = warp * 16;
-  if (!active) return;
-#pragma unroll
-  for (int half = 0; half < C::NB / 32; ++half) {
-    const int c0 = half * 32;
-    double x[2][4][2];
-    if (half == 0) {
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) x[mt][nt][0] = x[mt][nt][1] = 0.0;
-    } else {
-      // C2 -= X1 L21^T  (acc from the tile's C2, A = X1 (tile cols 0..31), B = inv[k][32+n])
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h)
-            x[mt][nt][h] = s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g];
-#pragma unroll
-      for (int k4 = 0; k4 < 8; ++k4) {
-        double fa[2], fb[4];
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.u.e.tile[k4 * 4 + q][r + mt * 8 + g];
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) fb[nt] = s.inv[k4 * 4 + q][32 + nt * 8 + g];
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-          for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
-      }
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g] = x[mt][nt][h];
-            x[mt][nt][h] = 0.0;
-          }
-      __syncwarp();
-    }
-    // X_half = C_half inv(L_half,half)^T
-#pragma unroll
-    for (int k4 = 0; k4 < 8; ++k4) {
-      double fa[2], fb[4];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt) fa[mt] = s.u.e.tile[c0 + k4 * 4 + q][r + mt * 8 + g];
-#pragma unroll
-      for (int nt = 0; nt < 4; ++nt) fb[nt] = s.inv[c0 + k4 * 4 + q][c0 + nt * 8 + g];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) dmma(x[mt][nt], fa[mt], fb[nt]);
-    }
-    __syncwarp();
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 4; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          s.u.e.tile[c0 + nt * 8 + 2 * q + h][r + mt * 8 + g] = x[mt][nt][h];
-    __syncwarp();
-  }
-}
-
-// Issue chunk kc (global ring index gi) with TMA bulk copies, by warp 0: lanes 0..KC-1
-// copy A column segments (rows r0..r0+ra-1), lanes 16..16+KC-1 the panel rows j0..j0+rb-1.
-// Segment lengths are rounded up to an even row count (16-byte multiple); the extra row is
-// padding (ldda even and > n when n is odd). Rows beyond are stale and only ever feed
-// output rows/columns that are never stored.
-template <class C>
-VB_DEVINL void issue_stage_bulk(BlockedSmem<C>& s, uint32_t gi, int kc, const double* A, int n,
-                                int ld, int r0, int j0, int lane) {
-  static_assert(C::KC <= 16, "one lane per column segment");
-  const int st = gi % C::STAGES;
-  const uint32_t u = gi / C::STAGES;
-  const int ra = (min(C::MB, n - r0) + 1) & ~1;
-  const int rb = (min(C::NB, n - j0) + 1) & ~1;
-  if (lane == 0) {
-    if (u > 0) mbar_wait(&s.empty[st], (u - 1) & 1);
-    mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * 8));
-  }
-  __syncwarp();
-  const int k0 = kc * C::KC;
-  if (lane < C::KC) {
-    bulk_g2s(&s.u.pipe.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * 8, &s.full[st]);
-  } else if (lane >= 16 && lane < 16 + C::KC) {
-    const int c = lane - 16;
-    bulk_g2s(&s.u.pipe.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * 8, &s.full[st]);
-  }
-}
-
-// One k-chunk of the panel update for this warp's tile: acc -= A_chunk B_chunk^T.
-template <class C>
-VB_DEVINL void mma_chunk(BlockedSmem<C>& s, int st, double (&acc)[C::MT][C::NT][2], int wrow,
-                         int wcol, int g, int q) {
-#pragma unroll
-  for (int kk = 0; kk < C::KC / 4; ++kk) {
-    double fa[C::MT], fb[C::NT];
-#pragma unroll
-    for (int mt = 0; mt < C::MT; ++mt) fa[mt] = -s.u.pipe.a[st][kk * 4 + q][wrow + mt * 8 + g];
-#pragma unroll
-    for (int nt = 0; nt < C::NT; ++nt) fb[nt] = s.u.pipe.b[st][kk * 4 + q][wcol + nt * 8 + g];
-#pragma unroll
-    for (int mt = 0; mt < C::MT; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < C::NT; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
-  }
-}
-
-// Blocked left-looking Cholesky of one matrix by the whole CTA.
-template <class C>
-VB_DEVINL void potrf_blocked_matrix(BlockedSmem<C>& s, double* __restrict__ A, int n, int ld,
-                                    int* info_out) {
-  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES;
-  constexpr int MT = C::MT, NT = C::NT;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int g = lane >> 2, q = lane & 3;
-  const int wrow = (warp % C::WARPS_M) * C::WM;  // warp's first row within the block
-  const int wcol = (warp / C::WARPS_M) * C::WN;  // warp's first panel column
-  // TMA bulk copies need 16-byte aligned column segments: even ldda and aligned base.
-  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
-  for (int j0 = 0; j0 < n; j0 += NB) {
-    const int nb = min(NB, n - j0);
-    const int nk = j0 / KC;
-    for (int r0 = j0; r0 < n; r0 += MB) {
-      const bool first = (r0 == j0);
-      const bool warp_active = (r0 + wrow) < n;
-      // ---- accumulators start from A's panel values (lower triangle only)
-      double acc[MT][NT][2];
-#pragma unroll
-      for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int row = r0 + wrow + mt * 8 + g, col = j0 + wcol + nt * 8 + 2 * q + h;
-            const bool v = row < n && col < j0 + nb && row >= col;
-            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
-          }
-      // ---- panel update on DMMA: acc -= L[r0:r0+MB, 0:j0] L[j0:j0+NB, 0:j0]^T
-      if (nk > 0) {
-        if (bulk) {
-          // TMA ring: warp 0 issues 1-D bulk copies of whole column segments into stage
-          // (chunk % STAGES); consumers wait on full[], release with one arrive per warp on
-          // empty[]; the producer waits on empty[] before refilling a stage.
-          const uint32_t gb = s.chunks;
-          if (warp == 0) {
-            fence_proxy_async();  // generic smem accesses (epilogue) before async writes
-            for (int p = 0; p < STAGES - 1 && p < nk; ++p)
-              issue_stage_bulk<C>(s, gb + p, p, A, n, ld, r0, j0, lane);
-          }
-          for (int kc = 0; kc < nk; ++kc) {
-            const uint32_t gi = gb + kc;
-            const int st = gi % STAGES;
-            if (warp == 0 && kc + STAGES - 1 < nk)
-              issue_stage_bulk<C>(s, gi + STAGES - 1, kc + STAGES - 1, A, n, ld, r0, j0, lane);
-            mbar_wait(&s.full[st], (gi / STAGES) & 1);
-            if (warp_active) mma_chunk<C>(s, st, acc, wrow, wcol, g, q);
-            fence_proxy_async();  // this thread's LDS of the slot before the TMA refill (WAR)
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&s.empty[st]);
-          }
-          __syncthreads();
-          if (tid == 0) s.chunks = gb + nk;
-        } else {
-#pragma unroll
-          for (int st = 0; st < STAGES - 1; ++st) {
-            if (st < nk) load_stage<C>(s, st, st, A, n, ld, r0, j0);
-            cp_async_commit();
-          }
-          for (int kc = 0; kc < nk; ++kc) {
-            cp_async_wait<STAGES - 2>();
-            __syncthreads();
-            const int pf = kc + STAGES - 1;
-            if (pf < nk) load_stage<C>(s, pf % STAGES, pf, A, n, ld, r0, j0);
-            cp_async_commit();
-            if (warp_active) mma_chunk<C>(s, kc % STAGES, acc, wrow, wcol, g, q);
-          }
-          cp_async_wait<0>();
-        }
-      }
-      __syncthreads();  // pipeline buffers are free: reuse as the C tile
-#pragma unroll
-      for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < NT; ++nt) {
-          const int r = wrow + mt * 8 + g, c = wcol + nt * 8 + 2 * q;
-          s.u.e.tile[c][r] = acc[mt][nt][0];
-          s.u.e.tile[c + 1][r] = acc[mt][nt][1];
-        }
-      __syncthreads();
-      if (first) {
-        const bool below = r0 + nb < n;
-        double* Ad = A + (size_t)j0 * ld + j0;
-        if constexpr (NB == 32) {
-          if (warp == 0) diag_block32(s, nb, lane, Ad, ld, below);
-        } else {
-          if (warp < 4) diag_block64(s, nb, warp, lane, Ad, ld, below);
-        }
-        fence_proxy_async();         // generic smem writes before the next TMA refill
-        fence_proxy_async_global();  // L11 stores before later TMA reads of them
-        __syncthreads();
-        if (s.info) {
-          if (tid == 0) *info_out = j0 + s.info;
-          return;
-        }
-        if (!below) continue;  // no rows below the diagonal block in this pass
-      }
-      // ---- panel factorize (TRSM) on DMMA, 32 columns at a time with 32x32 inverses:
-      //      X1 = C1 inv(L11)^T;  [NB=64: C2 -= X1 L21^T;  X2 = C2 inv(L22)^T]
-      //      Each warp owns 16 rows of the tile (reads and writes only its rows), so no CTA
-      //      barrier is needed between the steps.
-      trsm_rows16<C>(s, warp, lane,
-                     r0 + warp * 16 < n && !(first && warp * 16 + 16 <= nb));
-      __syncthreads();
-      const int row_lo = first ? j0 + nb : r0;
-      for (int idx = tid; idx < NB * MB; idx += C::THREADS) {
-        const int c = idx / MB, r = idx % MB;
-        const int row = r0 + r;
-        if (c < nb && row < n && row >= row_lo) A[(size_t)(j0 + c) * ld + row] = s.u.e.tile[c][r];
-      }
-      fence_proxy_async();         // generic smem accesses before the next TMA refill
-      fence_proxy_async_global();  // this panel's L stores before later TMA reads of them
-      __syncthreads();
-    }
-  }
-}
-
-// range: 0 (NB = 64) or 1 (NB = 32). wait_upstream: the kernel directly follows the scan.
-template <class C>
-__global__ void __launch_bounds__(C::THREADS, C::MINB)
-    potrf_blocked_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
-                         const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                         const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
-                         int wait_upstream) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  BlockedSmem<C>& s = *reinterpret_cast<BlockedSmem<C>*>(smem_raw);
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < C::STAGES; ++i) {
-      mbar_init(&s.full[i], 1);
-      mbar_init(&s.empty[i], C::THREADS / 32);
-    }
-    s.chunks = 0;
-    fence_proxy_async();  // make the initialised barriers visible to the async proxy
-  }
-  __syncthreads();
-  if (wait_upstream) pdl_wait();  // the scan's outputs (order, ctrl, info) are visible
-  pdl_launch_dependents();        // the next range's kernel may start filling freed SMs
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int tid = threadIdx.x;
-  for (;;) {
-    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
-    __syncthreads();
-    const int it = s.item;
-    __syncthreads();
-    if (it >= count) break;
-    const int m = order[start + it];
-    TL_BEGIN(t_tl)
-    potrf_blocked_matrix<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m);
-    __syncthreads();
-    TL_END(tid == 0, t_tl, m, 10 + range)
-  }
-}
-
 // =======================================================================================
-// v2 blocked kernel (large n): warp w owns 16 full rows of each 128-row block, so the TRSM
-// runs from registers and stores straight to global; the TMA stage ring is not aliased
-// with anything, so the producer (warp 0) keeps prefetching across the row blocks of a
-// panel; CTA-wide barriers only around the diagonal block and at the panel end.
+// Blocked kernel (n > ts) building blocks: warp w owns 16 full rows of each MB-row block, so
+// the TRSM runs from registers and stores straight to global; the TMA stage ring is not
+// aliased with anything, so the producer keeps prefetching across row blocks and panels.
 template <int NB_, int KC_, int STAGES_, int MINB_, int WARPS_ = 8>
 struct Cfg2 {
   static constexpr int NB = NB_, KC = KC_, STAGES = STAGES_, MINB = MINB_;
@@ -825,8 +402,6 @@ struct Cfg2 {
   static constexpr int THREADS = 32 * WARPS, MB = 16 * WARPS, NT = NB / 8;
   static constexpr int LDA = MB + 4, LDB = NB + 4, LDT = NB + 4;
 };
-using Cfg64b = Cfg2<64, 16, 3, 2>;
-using Cfg64c = Cfg2<64, 16, 3, 2, 7>;  // v3: 7 compute warps + 1 producer warp = 256 threads
 using Cfg64d = Cfg2<64, 16, 2, 3, 4>;  // v3, 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer
 
 template <class C>
@@ -1028,214 +603,6 @@ VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
       acc[mt][4 + nt][0] = x[mt][nt][0];
       acc[mt][4 + nt][1] = x[mt][nt][1];
     }
-}
-
-template <class C>
-VB_DEVINL void potrf_blocked2_matrix(Smem2<C>& s, double* __restrict__ A, int n, int ld,
-                                     int* info_out) {
-  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int g = lane >> 2, q = lane & 3;
-  const int wrow = warp * 16;
-  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
-  uint32_t gcons = s.chunks;  // ring position of the next chunk to consume (all threads)
-  for (int j0 = 0; j0 < n; j0 += NB) {
-    const int nb = min(NB, n - j0);
-    const int nk = j0 / KC;
-    // producer state (meaningful in warp 0): next chunk of this panel to issue
-    int p_r0 = j0, p_kc = 0;
-    uint32_t gprod = gcons;
-    auto produce = [&]() {
-      if (p_r0 < n && nk > 0) {
-        issue_chunk2<C>(s, gprod, p_kc, A, n, ld, p_r0, j0, lane, bulk);
-        ++gprod;
-        if (++p_kc == nk) {
-          p_kc = 0;
-          p_r0 += MB;
-        }
-      }
-    };
-    if (warp == 0) {
-      fence_proxy_async();
-      for (int i = 0; i < STAGES - 1; ++i) produce();
-    }
-    for (int r0 = j0; r0 < n; r0 += MB) {
-      const bool first = (r0 == j0);
-      const bool active = (r0 + wrow) < n;
-      VB_T0(t_a)
-      double acc[2][NT][2];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
-            const bool v = row < n && col < j0 + nb && row >= col;
-            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
-          }
-      VB_ADD(5, t_a)
-      if (warp == 0 && lane < NB && bulk && r0 + MB < n) {
-        // warm L2 with the next row block's panel values (the accumulators' start)
-        const int rn = (min(MB, n - r0 - MB) + 1) & ~1;
-        if (lane < nb) bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0 + MB, rn * 8);
-      }
-      // columns this warp must compute: in the first row block the diagonal-block warps skip
-      // the tiles strictly above the diagonal (SYRK); warp-uniform bound
-#ifndef VB_V2_SKIP
-#define VB_V2_SKIP 0
-#endif
-      const int ntl = (VB_V2_SKIP && first && wrow < NB) ? (wrow + 16) / 8 : NT;
-      VB_T0(t_k)
-      for (int kc = 0; kc < nk; ++kc) {
-        if (warp == 0) produce();
-        const uint32_t gi = gcons + kc;
-        const int st = gi % STAGES;
-        mbar_wait(&s.full[st], (gi / STAGES) & 1);
-        if (active) {
-#pragma unroll
-          for (int kk = 0; kk < KC / 4; ++kk) {
-            double fa[2], fb[NT];
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
-#pragma unroll
-            for (int nt = 0; nt < NT; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-              for (int nt = 0; nt < NT; ++nt)
-                if (nt < ntl) dmma(acc[mt][nt], fa[mt], fb[nt]);
-          }
-        }
-        fence_proxy_async();  // this thread's LDS of the slot before the TMA refill (WAR)
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&s.empty[st]);
-      }
-      gcons += nk;
-      VB_ADD(0, t_k)
-      VB_T0(t_d)
-      if (first) {
-        // Diagonal-block warps hand their accumulators to smem and factor the block; the
-        // other warps wait for inv(L) and do their TRSM. Two separate branches joined only by
-        // named barriers, so no accumulator is live across the out-of-line diagonal call.
-        const bool below = r0 + nb < n;
-        const bool diag_warp = warp < NB / 16;  // this warp's 16 rows are diagonal-block rows
-        bool failed;
-        if (diag_warp) {
-#pragma unroll
-          for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-            for (int nt = 0; nt < NT; ++nt) {
-              s.T[nt * 8 + 2 * q][wrow + mt * 8 + g] = acc[mt][nt][0];
-              s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
-            }
-          bar_group(2, C::THREADS);
-          diag_block64v2(s, nb, warp, lane, A + (size_t)j0 * ld + j0, ld, below);
-          bar_group(3, C::THREADS);
-          failed = s.info != 0;
-        } else {
-          bar_group(2, C::THREADS);
-          bar_group(3, C::THREADS);
-          failed = s.info != 0;
-          if (!failed && below && active) {
-            trsm_regs64(s, acc, lane);
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-              for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                  const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
-                  if (row < n && row >= j0 + nb && col < nb)
-                    A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
-                }
-          }
-        }
-        VB_ADD(1, t_d)
-        if (failed) {
-          if (tid == 0) *info_out = j0 + s.info;
-          // consume the chunks the producer already issued for this panel so the ring stays
-          // consistent for the next matrix
-          if (warp == 0) {
-            for (uint32_t gi = gcons; gi < gprod; ++gi) {
-              const int st = gi % STAGES;
-              if (lane == 0) mbar_wait(&s.full[st], (gi / STAGES) & 1);
-            }
-          }
-          __syncthreads();
-          if (warp == 0 && lane == 0) {
-            for (uint32_t gi = gcons; gi < gprod; ++gi)
-              for (int w = 0; w < C::WARPS; ++w) mbar_arrive(&s.empty[gi % STAGES]);
-          }
-          const uint32_t done = __shfl_sync(kFull, gprod, 0);
-          if (tid == 0) s.chunks = done;
-          __syncthreads();
-          return;
-        }
-        continue;
-      }
-      VB_T0(t_t)
-      // ---- TRSM in registers + direct stores of the rows below the diagonal block
-      if (active) {
-        trsm_regs64(s, acc, lane);
-        const int row_lo = r0;
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-          for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
-              if (row < n && row >= row_lo && col < nb)
-                A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
-            }
-      }
-      VB_ADD(2, t_t)
-    }
-    // panel end: every L value of this panel is stored before the next panel's TMA reads
-    VB_T0(t_p)
-    fence_proxy_async_global();
-    __syncthreads();
-    VB_ADD(3, t_p)
-  }
-  if (tid == 0) s.chunks = gcons;
-  __syncthreads();
-}
-
-template <class C>
-__global__ void __launch_bounds__(C::THREADS, C::MINB)
-    potrf_blocked2_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
-                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                          const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
-                          int range, int wait_upstream) {
-  extern __shared__ __align__(128) unsigned char smem_raw2[];
-  Smem2<C>& s = *reinterpret_cast<Smem2<C>*>(smem_raw2);
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < C::STAGES; ++i) {
-      mbar_init(&s.full[i], 1);
-      mbar_init(&s.empty[i], C::WARPS);
-    }
-    s.chunks = 0;
-    fence_proxy_async();
-  }
-  __syncthreads();
-  if (wait_upstream) pdl_wait();
-  pdl_launch_dependents();
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int tid = threadIdx.x;
-  for (;;) {
-    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
-    __syncthreads();
-    const int it = s.item;
-    __syncthreads();
-    if (it >= count) break;
-    const int m = order[start + it];
-    VB_T0(t_m)
-    potrf_blocked2_matrix<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m);
-    VB_ADD(4, t_m)
-  }
 }
 
 // =======================================================================================
@@ -1489,337 +856,6 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     }
     TL_END(tid == 0, t_tl, m, 30)
   }
-}
-
-// =======================================================================================
-// v4 "team" kernel (large n): one CTA per SM = three independent matrix teams plus one diagonal
-// warp. Measured on B200 (tools/contention_bench.cu): a warp issuing back-to-back DMMAs starves
-// every other FP64 instruction (DFMA, DMUL and even dependent DMMAs) on the same SM sub-partition
-// — a 256-long DFMA chain takes 60x longer next to one DMMA-issuing warp and ~3700x next to two —
-// while FP32, integer and MUFU instructions are unaffected. In the v3 kernel the POTF2/TRTRI chain
-// of one CTA shares its sub-partitions with the other CTAs' k-loops, so the diagonal phase takes
-// 46 K cycles per 64x64 block under load instead of 21 K alone (25-30 % of a CTA's time for
-// n <= 512). Here the roles are pinned to sub-partitions (warp w runs on SMSP w % 4):
-//   SMSPs 0-2: 12 consumer warps, 4 per team (16 rows each of the team's 64-row blocks);
-//   SMSP 3:    one TMA producer warp per team (warps 3, 7, 11) and the diagonal warp (15),
-//              which factors every team's 64x64 diagonal blocks with no DMMA stream beside it.
-// The consumers hand the diagonal tile over (tile_ready mbarrier) and go straight on with the next
-// row block's panel update (look-ahead); they wait for the factor (diag_done) only before their
-// first TRSM of the panel.
-constexpr int kTeams = 3;
-constexpr int kTeamWarps = 16;
-
-struct TeamCtl {
-  uint64_t tile_ready;  // 4 consumer-warp arrivals per panel: the diagonal tile is in s.T
-  uint64_t diag_done;   // 1 arrival (diagonal warp): L11/L21/L22 stored, inverses in s.T, s.info
-  double* A;            // request: the matrix and its panel
-  int* info_out;
-  int ld, j0, nb, below;
-  int item;
-  volatile int done;  // the team has no more matrices
-};
-
-template <class C>
-struct alignas(128) TeamSlot {  // 128-byte aligned: the TMA destinations inside stay aligned
-  Smem2<C> s;
-};
-template <class C>
-struct TeamSmem {
-  TeamSlot<C> team[kTeams];
-  TeamCtl ctl[kTeams];
-};
-
-// Diagonal 64x64 block by ONE warp (same factorisation as diag_block64v2):
-//   L11 = potf2(C11), inv(L11) -> T12 slot; L21 = C21 inv(L11)^T -> T21 (and global);
-//   C22 -= L21 L21^T; L22 = potf2(C22), inv(L22) -> T11 slot. Sets s.info (in-block, 1-based).
-template <class CC>
-__device__ __noinline__ void diag_block64_1w(Smem2<CC>& s, int nb, int lane, double* Ad, int ld,
-                                             bool below) {
-  constexpr int LDT = CC::LDT;
-  double* T = &s.T[0][0];
-  double* INV11 = T + 32 * LDT;
-  double* INV22 = T;
-  const int g = lane >> 2, q = lane & 3;
-  const int nb1 = min(nb, 32), nb2 = nb - nb1;
-  int info = potf2_block32(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
-  if (info || nb2 <= 0) {
-    if (lane == 0) s.info = info;
-    __syncwarp();
-    return;
-  }
-  trtri32_dmma_warp(T, LDT, s.tv, INV11, LDT, s.S, LDS_T, lane);
-  {  // L21 = C21 inv(L11)^T: all four quarters in registers before T21 is overwritten
-    double acc[4][2][2][2];
-#pragma unroll
-    for (int wg = 0; wg < 4; ++wg)
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 2; ++nt) acc[wg][mt][nt][0] = acc[wg][mt][nt][1] = 0.0;
-#pragma unroll
-    for (int wg = 0; wg < 4; ++wg)
-      mm32_quarter(acc[wg], wg, lane, [&](int m, int k) { return T[k * LDT + 32 + m]; },
-                   [&](int k, int n) { return INV11[k * LDT + n]; });
-    __syncwarp();
-#pragma unroll
-    for (int wg = 0; wg < 4; ++wg) {
-      const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
-            T[c * LDT + r] = acc[wg][mt][nt][h];
-            if (r < nb) Ad[(size_t)c * ld + r] = acc[wg][mt][nt][h];
-          }
-    }
-  }
-  __syncwarp();
-  // C22 -= L21 L21^T on the three quarters on or below the diagonal (reads T21, writes T22)
-#pragma unroll
-  for (int wg = 0; wg < 4; ++wg) {
-    if (wg == 1) continue;
-    const int m0 = (wg >> 1) * 16, n0 = (wg & 1) * 16;
-    double acc[2][2][2];
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          acc[mt][nt][h] = T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g];
-    mm32_quarter(acc, wg, lane, [&](int m, int k) { return -T[k * LDT + 32 + m]; },
-                 [&](int k, int n) { return T[k * LDT + 32 + n]; });
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          T[(32 + n0 + nt * 8 + 2 * q + h) * LDT + 32 + m0 + mt * 8 + g] = acc[mt][nt][h];
-  }
-  __syncwarp();
-  double* T22 = T + 32 * LDT + 32;
-  info = potf2_block32(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf, s.sv + 32,
-                       s.tv + 32);
-  if (!info && below) trtri32_dmma_warp(T22, LDT, s.tv + 32, INV22, LDT, s.S, LDS_T, lane);
-  if (lane == 0) s.info = info ? 32 + info : 0;
-  __syncwarp();
-}
-
-VB_DEVINL bool mbar_test(uint64_t* bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-      " selp.u32 %0, 1, 0, p;\n}\n"
-      : "=r"(ok)
-      : "r"(smem_u32(bar)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-
-// Team consumer warp cw (0..3, rows 16cw..16cw+15 of each 64-row block) of one matrix.
-template <class C>
-VB_DEVINL void consume_matrix4(Smem2<C>& s, TeamCtl& x, double* __restrict__ A, int n, int ld,
-                               int* info_out, uint32_t& gchunk, uint32_t& gdiag, int cw, int lane,
-                               int cbar) {
-  constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
-  static_assert(MB == NB, "the first row block of a panel is exactly its diagonal block");
-  const int g = lane >> 2, q = lane & 3;
-  const int wrow = cw * 16;
-  for (int j0 = 0; j0 < n; j0 += NB) {
-    const int nb = min(NB, n - j0);
-    const int nk = j0 / KC;
-    bool failed = false, waited = false;
-    for (int r0 = j0; r0 < n; r0 += MB) {
-      const bool first = (r0 == j0);
-      const bool active = (r0 + wrow) < n;
-      if (failed) {  // drain this panel's remaining chunks (already issued by the producer)
-        for (int kc = 0; kc < nk; ++kc) {
-          const uint32_t gi = gchunk++;
-          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
-        }
-        continue;
-      }
-      double acc[2][NT][2];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
-            const bool v = row < n && col < j0 + nb && row >= col;
-            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
-          }
-      const int ntl = first ? (wrow + 16) / 8 : NT;
-      if (!active) {
-        k_loop3<C, 0>(s, acc, gchunk, nk, wrow, lane);
-      } else if (ntl == 2) {
-        k_loop3<C, 2>(s, acc, gchunk, nk, wrow, lane);
-      } else if (ntl == 4) {
-        k_loop3<C, 4>(s, acc, gchunk, nk, wrow, lane);
-      } else if (ntl == 6) {
-        k_loop3<C, 6>(s, acc, gchunk, nk, wrow, lane);
-      } else {
-        k_loop3<C, NT>(s, acc, gchunk, nk, wrow, lane);
-      }
-      if (first) {  // hand the diagonal tile to the diagonal warp; go on with the next block
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-          for (int nt = 0; nt < NT; ++nt) {
-            s.T[nt * 8 + 2 * q][wrow + mt * 8 + g] = acc[mt][nt][0];
-            s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
-          }
-        if (cw == 0 && lane == 0) {
-          x.A = A;
-          x.info_out = info_out;
-          x.ld = ld;
-          x.j0 = j0;
-          x.nb = nb;
-          x.below = (j0 + nb < n) ? 1 : 0;
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&x.tile_ready);
-        continue;
-      }
-      if (!waited) {  // the first TRSM of the panel needs the diagonal factor
-        mbar_wait(&x.diag_done, gdiag & 1);
-        waited = true;
-        failed = s.info != 0;
-        if (failed) continue;
-      }
-      if (active) {
-        trsm_regs64(s, acc, lane);
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-          for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
-              if (row < n && col < nb) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
-            }
-      }
-    }
-    if (!waited) {
-      mbar_wait(&x.diag_done, gdiag & 1);
-      failed = s.info != 0;
-    }
-    ++gdiag;
-    // panel end: this warp's L stores are fenced for the async proxy and released to the
-    // producer (the diagonal warp fenced the diagonal block's stores before diag_done)
-    fence_proxy_async_global();
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&s.panel_done);
-    if (failed) {
-      if (j0 + NB < n) {  // the next panel's independent chunks the producer already issued
-        for (int kc = 0; kc < nk; ++kc) {
-          const uint32_t gi = gchunk++;
-          mbar_wait(&s.full[gi % STAGES], (gi / STAGES) & 1);
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&s.empty[gi % STAGES]);
-        }
-      }
-      break;
-    }
-    bar_group(cbar, 128);  // every TRSM read of s.T is done before the next tile is written
-  }
-}
-
-template <class C>
-__global__ void __launch_bounds__(32 * kTeamWarps, 1)
-    potrf_team_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
-                      const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                      const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
-                      int wait_upstream) {
-  extern __shared__ __align__(128) unsigned char smem_raw4[];
-  TeamSmem<C>& S = *reinterpret_cast<TeamSmem<C>*>(smem_raw4);
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  if (tid < kTeams) {
-    Smem2<C>& s = S.team[tid].s;
-    for (int i = 0; i < C::STAGES; ++i) {
-      mbar_init(&s.full[i], 1);
-      mbar_init(&s.empty[i], 4);
-    }
-    mbar_init(&s.panel_done, 4);
-    s.info = 0;
-    mbar_init(&S.ctl[tid].tile_ready, 4);
-    mbar_init(&S.ctl[tid].diag_done, 1);
-    S.ctl[tid].done = 0;
-    fence_proxy_async();
-  }
-  __syncthreads();
-  if (wait_upstream) pdl_wait();
-  pdl_launch_dependents();
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int sp = warp & 3;
-  if (warp == kTeamWarps - 1) {
-    // ---- diagonal warp: serve the teams' diagonal tiles as they become ready
-    uint32_t par[kTeams] = {0, 0, 0};
-    bool live[kTeams] = {true, true, true};
-    int nlive = kTeams;
-    while (nlive > 0) {
-      bool did = false;
-#pragma unroll
-      for (int t = 0; t < kTeams; ++t) {
-        if (!live[t]) continue;
-        TeamCtl& x = S.ctl[t];
-        if (mbar_test(&x.tile_ready, par[t])) {
-          par[t] ^= 1;
-          Smem2<C>& s = S.team[t].s;
-          double* Ad = x.A + (size_t)x.j0 * x.ld + x.j0;
-          diag_block64_1w(s, x.nb, lane, Ad, x.ld, x.below != 0);
-          if (s.info && lane == 0) *x.info_out = x.j0 + s.info;
-          fence_proxy_async_global();  // the diagonal block's L stores before later TMA reads
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&x.diag_done);
-          did = true;
-        } else if (x.done) {
-          live[t] = false;
-          --nlive;
-        }
-      }
-      if (!did) __nanosleep(32);
-    }
-    return;
-  }
-  int team, cw = -1;
-  if (sp == 3) {
-    team = warp >> 2;  // producers: warps 3, 7, 11
-  } else {
-    const int c = (warp >> 2) * 3 + sp;
-    team = c >> 2;
-    cw = c & 3;
-  }
-  Smem2<C>& s = S.team[team].s;
-  TeamCtl& x = S.ctl[team];
-  const int tbar = 1 + 2 * team, cbar = 2 + 2 * team;  // team (160 threads) / consumers (128)
-  uint32_t gchunk = 0, gpanel = 0, gdiag = 0;
-  for (;;) {
-    if (cw == 0 && lane == 0) x.item = atomicAdd(&ctrl->head[range], 1);
-    bar_group(tbar, 160);
-    const int it = x.item;
-    bar_group(tbar, 160);
-    if (it >= count) break;
-    const int m = order[start + it];
-    TL_BEGIN(t_tl)
-    if (cw < 0) {
-      produce_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
-    } else {
-      consume_matrix4<C>(s, x, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gdiag, cw, lane,
-                         cbar);
-    }
-    TL_END(cw == 0 && lane == 0, t_tl, m, 50)
-  }
-  if (cw == 0 && lane == 0) x.done = 1;
 }
 
 // =======================================================================================
@@ -2170,12 +1206,12 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
   __shared__ WarpSmem s;
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
   if (wait_upstream) pdl_wait();
-  const int start = *(volatile const int*)&ctrl->start[3];
-  const int count = *(volatile const int*)&ctrl->count[3];
+  const int start = *(volatile const int*)&ctrl->start[2];
+  const int count = *(volatile const int*)&ctrl->count[2];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   for (;;) {
     int w = 0;
-    if (lane == 0) w = atomicAdd(&ctrl->head[3], 1);
+    if (lane == 0) w = atomicAdd(&ctrl->head[2], 1);
     w = __shfl_sync(kFull, w, 0);
     if (w >= count) break;
     const int m = order[start + w];
@@ -2220,14 +1256,14 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 
 // ---------------------------------------------------------------------------------------
 static int g_num_sms = 0;
-static int g_occ32 = 0, g_occ64 = 0, g_occ64b = 0, g_occ64c = 0, g_occ64d = 0;
-static int g_v3w = 4;
-static int g_t64 = -1;
+static int g_occ64 = 0;
 static int g_ts = -1;
 static int g_occ_small = 0, g_occ_wsmall = 0;
 static int g_small = -1;
-static int g_v2 = -1;
 
+// Size threshold: n > ts takes the blocked NB=64 kernel, 32 < n <= ts the small-matrix kernel
+// (env VB_TS; default 128, measured: the blocked kernel beats the small kernel above 128 and
+// loses below, tools/cfgtime.py sweeps in profiles/r01).
 int potrf_ts() {
   if (g_ts < 0) {
     const char* e = getenv("VB_TS");
@@ -2235,66 +1271,6 @@ int potrf_ts() {
     if (g_ts < kWarpMaxN) g_ts = kWarpMaxN;
   }
   return g_ts;
-}
-
-int potrf_t64() {
-  if (g_t64 < 0) {
-    const char* e = getenv("VB_T64");
-    g_t64 = e ? atoi(e) : 256;
-    if (g_t64 < kWarpMaxN) g_t64 = kWarpMaxN;
-  }
-  return g_t64;
-}
-
-template <class C>
-static cudaError_t setup_kernel(int* occ) {
-  cudaError_t e = cudaFuncSetAttribute(potrf_blocked_kernel<C>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)sizeof(BlockedSmem<C>));
-  if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked_kernel<C>, C::THREADS,
-                                                    sizeof(BlockedSmem<C>));
-  if (*occ < 1) *occ = 1;
-  return e;
-}
-
-template <class C>
-static cudaError_t setup_v3(int* occ) {
-  cudaError_t e = cudaFuncSetAttribute(potrf_blocked3_kernel<C>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)sizeof(Smem2<C>));
-  if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked3_kernel<C>,
-                                                    32 * (C::WARPS + 1), sizeof(Smem2<C>));
-  if (*occ < 1) *occ = 1;
-  return e;
-}
-
-static int g_v4 = -1;
-static bool g_team_ok = false;
-
-template <class C>
-static cudaError_t setup_team() {
-  cudaError_t e = cudaFuncSetAttribute(potrf_team_kernel<C>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)sizeof(TeamSmem<C>));
-  if (e != cudaSuccess) return e;
-  int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, potrf_team_kernel<C>, 32 * kTeamWarps,
-                                                    sizeof(TeamSmem<C>));
-  g_team_ok = (e == cudaSuccess && occ == 1);
-  return e;
-}
-
-template <class C>
-static cudaError_t launch_v3(cudaLaunchConfig_t& cfg, int occ, int batch, const int* d_n,
-                             double* const* dA, const int* d_ldda, int* d_info, const Ctrl* ctrl,
-                             const int* order, int range, int wait) {
-  cfg.blockDim = dim3(32 * (C::WARPS + 1));
-  cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * occ)));
-  cfg.dynamicSmemBytes = sizeof(Smem2<C>);
-  return cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel<C>, d_n, dA, d_ldda, d_info, ctrl, order,
-                            range, wait);
 }
 
 static cudaError_t init_device_info() {
@@ -2305,30 +1281,13 @@ static cudaError_t init_device_info() {
   int sms = 0;
   e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
-  if ((e = setup_kernel<Cfg32>(&g_occ32)) != cudaSuccess) return e;
-  if ((e = setup_kernel<Cfg64>(&g_occ64)) != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(potrf_blocked2_kernel<Cfg64b>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64b>));
+  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64d>));
   if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64b, potrf_blocked2_kernel<Cfg64b>,
-                                                    Cfg64b::THREADS, sizeof(Smem2<Cfg64b>));
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64, potrf_blocked3_kernel<Cfg64d>,
+                                                    32 * (Cfg64d::WARPS + 1), sizeof(Smem2<Cfg64d>));
   if (e != cudaSuccess) return e;
-  if (g_occ64b < 1) g_occ64b = 1;
-  if ((e = setup_v3<Cfg64c>(&g_occ64c)) != cudaSuccess) return e;
-  if ((e = setup_v3<Cfg64d>(&g_occ64d)) != cudaSuccess) return e;
-  if ((e = setup_team<Cfg64d>()) != cudaSuccess) return e;
-  {
-    const char* v = getenv("VB_V4");
-    g_v4 = v ? atoi(v) : 0;
-  }
-  {
-    const char* v = getenv("VB_V3W");
-    g_v3w = v ? atoi(v) : 4;
-  }
-  {
-    const char* v = getenv("VB_V2");
-    g_v2 = v ? atoi(v) : 3;
-  }
+  if (g_occ64 < 1) g_occ64 = 1;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_kernel,
                                                     32 * kSmallWarps, 0);
   if (e != cudaSuccess) return e;
@@ -2341,11 +1300,13 @@ static cudaError_t init_device_info() {
     g_small = v ? atoi(v) : 2;
   }
   potrf_ts();
-  potrf_t64();
   g_num_sms = sms;
   return cudaSuccess;
 }
 
+// One persistent grid per non-empty size range, chained with programmatic dependent launch
+// (each grid releases the next as soon as it starts, so the next range's CTAs take the SMs
+// the previous kernel frees at its tail).
 cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
                                cudaStream_t stream) {
@@ -2359,41 +1320,12 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.numAttrs = 1;
   cfg.stream = stream;
   int wait = 1;  // the first factorisation kernel after the scan waits for it
-  if (max_n_hint > g_t64) {
-    if (g_v2 == 3) {
-      if (g_v4 && g_team_ok) {
-        cfg.blockDim = dim3(32 * kTeamWarps);
-        cfg.gridDim = dim3(std::max(1, std::min((batch + kTeams - 1) / kTeams, g_num_sms)));
-        cfg.dynamicSmemBytes = sizeof(TeamSmem<Cfg64d>);
-        e = cudaLaunchKernelEx(&cfg, potrf_team_kernel<Cfg64d>, d_n, dA, d_ldda, d_info, ctrl,
-                               order, 0, wait);
-      } else if (g_v3w == 4) {
-        e = launch_v3<Cfg64d>(cfg, g_occ64d, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
-      } else {
-        e = launch_v3<Cfg64c>(cfg, g_occ64c, batch, d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
-      }
-    } else if (g_v2) {
-      cfg.blockDim = dim3(Cfg64b::THREADS);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64b)));
-      cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64b>);
-      e = cudaLaunchKernelEx(&cfg, potrf_blocked2_kernel<Cfg64b>, d_n, dA, d_ldda, d_info, ctrl,
-                             order, 0, wait);
-    } else {
-      cfg.blockDim = dim3(Cfg64::THREADS);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
-      cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg64>);
-      e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg64>, d_n, dA, d_ldda, d_info, ctrl,
-                             order, 0, wait);
-    }
-    if (e != cudaSuccess) return e;
-    wait = 0;
-  }
-  if (max_n_hint > g_ts && g_ts < g_t64) {
-    cfg.blockDim = dim3(Cfg32::THREADS);
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ32)));
-    cfg.dynamicSmemBytes = sizeof(BlockedSmem<Cfg32>);
-    e = cudaLaunchKernelEx(&cfg, potrf_blocked_kernel<Cfg32>, d_n, dA, d_ldda, d_info, ctrl, order,
-                           1, wait);
+  if (max_n_hint > g_ts) {
+    cfg.blockDim = dim3(32 * (Cfg64d::WARPS + 1));
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
+    cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64d>);
+    e = cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel<Cfg64d>, d_n, dA, d_ldda, d_info, ctrl,
+                           order, 0, wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
@@ -2402,13 +1334,13 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
       cfg.blockDim = dim3(32 * kSmallWarps);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
       cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
+      e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 1,
                              wait);
     } else {
       cfg.blockDim = dim3(32);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
       cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, potrf_wsmall_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 2,
+      e = cudaLaunchKernelEx(&cfg, potrf_wsmall_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 1,
                              wait);
     }
     if (e != cudaSuccess) return e;
@@ -2424,17 +1356,16 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
 
 void potrf_occupancy(int* out4) {
   init_device_info();
-  out4[0] = g_v3w == 4 ? g_occ64d : g_occ64c;
-  out4[1] = g_v3w == 4 ? Cfg64d::WARPS : Cfg64c::WARPS;
-  out4[2] = g_occ32;
+  out4[0] = g_occ64;
+  out4[1] = Cfg64d::WARPS;
+  out4[2] = 0;  // (no separate NB=32 range)
   out4[3] = g_small == 2 ? g_occ_small : g_occ_wsmall;
 }
 
 int potrf_num_launches(int max_n_hint) {
   init_device_info();
   if (max_n_hint <= kWarpMaxN) return 1;  // direct warp kernel only
-  const int t64 = potrf_t64(), ts = potrf_ts();
-  return 3 + (max_n_hint > ts && ts < t64 ? 1 : 0) + (max_n_hint > t64 ? 1 : 0);
+  return 3 + (max_n_hint > potrf_ts() ? 1 : 0);
 }
 
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,

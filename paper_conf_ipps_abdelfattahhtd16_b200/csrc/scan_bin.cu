@@ -20,8 +20,8 @@ constexpr int kKeys = 4096;  // sort keys: min(n, kKeys-1) (larger n share the t
 
 __global__ void __launch_bounds__(kScanThreads, 1)
     scan_bin_kernel(const int* __restrict__ d_n, const int* __restrict__ d_ldda,
-                    int* __restrict__ d_info, int batch, int max_n, int check_max, int t64,
-                    int ts, Ctrl* __restrict__ ctrl, int* __restrict__ order) {
+                    int* __restrict__ d_info, int batch, int max_n, int check_max, int ts,
+                    Ctrl* __restrict__ ctrl, int* __restrict__ order) {
   // Let the dependent (factorisation) grid launch and reach its griddepcontrol.wait now.
   pdl_launch_dependents();
   __shared__ int hist[kKeys];
@@ -86,12 +86,9 @@ __global__ void __launch_bounds__(kScanThreads, 1)
   }
   __syncthreads();
   if (tid == 0) {
-    // start[k] = #items with key > k (descending order): the four ranges are contiguous.
-    auto clampk = [](int t) { return t < kWarpMaxN ? kWarpMaxN : (t > kKeys - 1 ? kKeys - 1 : t); };
-    const int tk64 = clampk(t64);
-    const int tks = clampk(ts < t64 ? ts : t64);
-    const int b0 = hist[tk64], b1 = hist[tks], b2 = hist[kWarpMaxN], b3 = hist[0];
-    const int bounds[kRanges + 1] = {0, b0, b1, b2, b3};
+    // start[k] = #items with key > k (descending order): the three ranges are contiguous.
+    const int tks = ts < kWarpMaxN ? kWarpMaxN : (ts > kKeys - 1 ? kKeys - 1 : ts);
+    const int bounds[kRanges + 1] = {0, hist[tks], hist[kWarpMaxN], hist[0]};
     for (int r = 0; r < kRanges; ++r) {
       ctrl->head[r] = 0;
       ctrl->start[r] = bounds[r];
@@ -113,7 +110,7 @@ __global__ void __launch_bounds__(kScanThreads, 1)
 cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int batch, int max_n,
                             bool check_max, Ctrl* ctrl, int* order, cudaStream_t stream) {
   scan_bin_kernel<<<1, kScanThreads, 0, stream>>>(d_n, d_ldda, d_info, batch, max_n,
-                                                  check_max ? 1 : 0, potrf_t64(), potrf_ts(), ctrl, order);
+                                                  check_max ? 1 : 0, potrf_ts(), ctrl, order);
   return cudaGetLastError();
 }
 

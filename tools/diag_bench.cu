@@ -9,7 +9,7 @@ using namespace vb;
 __global__ void __launch_bounds__(256) diag_kernel(double* gA, int ld, int reps, long long* out,
                                                    int which) {
   extern __shared__ __align__(128) unsigned char sm[];
-  Smem2<Cfg64c>& s = *reinterpret_cast<Smem2<Cfg64c>*>(sm);
+  Smem2<Cfg64d>& s = *reinterpret_cast<Smem2<Cfg64d>*>(sm);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   long long t_tot = 0;
   for (int it = 0; it < reps; ++it) {
@@ -21,12 +21,12 @@ __global__ void __launch_bounds__(256) diag_kernel(double* gA, int ld, int reps,
     __syncthreads();
     long long t0 = clock64();
     if (which == 0) {
-      if (warp == 0) potf2_block32(&s.T[0][0], Cfg64c::LDT, 32, lane, gA, ld, s.wbuf, s.sv, s.tv);
+      if (warp == 0) potf2_block32(&s.T[0][0], Cfg64d::LDT, 32, lane, gA, ld, s.wbuf, s.sv, s.tv);
     } else if (which == 1) {
       if (warp == 0) {
-        potf2_block32(&s.T[0][0], Cfg64c::LDT, 32, lane, gA, ld, s.wbuf, s.sv, s.tv);
+        potf2_block32(&s.T[0][0], Cfg64d::LDT, 32, lane, gA, ld, s.wbuf, s.sv, s.tv);
         t0 = clock64();
-        trtri32_dmma_warp(&s.T[0][0], Cfg64c::LDT, s.tv, &s.T[32][0], Cfg64c::LDT, s.S, LDS_T, lane);
+        trtri32_dmma_warp(&s.T[0][0], Cfg64d::LDT, s.tv, &s.T[32][0], Cfg64d::LDT, s.S, LDS_T, lane);
       }
     } else {
       if (warp < 4) diag_block64v2(s, 64, warp, lane, gA, ld, true);
@@ -62,7 +62,7 @@ __global__ void __launch_bounds__(256) hog_kernel(double* sink, int iters) {
 int main() {
   double* gA; long long* out; double* sink;
   cudaMalloc(&gA, 64 * 64 * 8 * 4); cudaMalloc(&out, 8 * 1024); cudaMalloc(&sink, 64);
-  int smem = sizeof(Smem2<Cfg64c>);
+  int smem = sizeof(Smem2<Cfg64d>);
   cudaFuncSetAttribute(diag_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   const char* names[3] = {"potf2_block32", "trtri32", "diag_block64v2"};
   for (int which = 0; which < 3; ++which) {
