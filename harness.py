@@ -34,19 +34,22 @@ class DeviceBatch:
         self.d_gidx = torch.from_numpy(self.gidx).to(self.device)
         self.d_info = torch.full((max(self.B, 1),), -12345, dtype=torch.int32, device=self.device)
 
-    def fill(self, poison=False, stream=None):
+    def fill(self, poison=False, stream=None, uplo="L"):
         s = torch.cuda.current_stream().cuda_stream if stream is None else stream
+        flags = (1 if poison else 0) | (2 if uplo == "U" else 0)
         vbdev.fill_f1(self.seed, self.B, self.d_n.data_ptr(), self.d_ldda.data_ptr(),
-                      self.d_ptrs.data_ptr(), self.d_gidx.data_ptr(), self.nonspd_mod, poison, s)
+                      self.d_ptrs.data_ptr(), self.d_gidx.data_ptr(), self.nonspd_mod, flags, s)
         return self
 
-    def set_matrix(self, i, A: np.ndarray, poison=True):
-        """Write a host matrix (full n x n; only what the ldda block holds) into slot i."""
+    def set_matrix(self, i, A: np.ndarray, poison=True, uplo="L"):
+        """Write a host matrix into slot i: its lower ('L') or upper ('U') triangle; the other
+        strict triangle and the padding rows get the NaN poison."""
         n, ld = int(self.n[i]), int(self.ldda[i])
         blk = np.full((ld, n), np.nan)
         if poison:
             blk.view(np.uint64)[:] = np.uint64(vbgen.NAN_POISON_BITS)
-        blk[:n, :n] = np.where(np.tril(np.ones((n, n), bool)), A, blk[:n, :n])
+        tri = np.tril(np.ones((n, n), bool)) if uplo == "L" else np.triu(np.ones((n, n), bool))
+        blk[:n, :n] = np.where(tri, A, blk[:n, :n])
         t = torch.from_numpy(blk.ravel(order="F").copy())
         self.arena[self.off[i]: self.off[i] + ld * n].copy_(t)
 

@@ -41,8 +41,12 @@ typedef struct CUstream_st* vb_stream_t; /* == cudaStream_t */
  * -> panel factorize (trsm)); PAPER.md:724-812 (§III-E separated kernels); error reporting
  * follows LAPACK DPOTRF [7] (PAPER.md:2291-2297 lists it as future work).
  *
- *  uplo       'L' (lower) — the factor L overwrites the lower triangle of each A_i.
- *             'U' is not yet supported and returns -1.
+ *  uplo       'L' (lower): A_i = L L^T, the factor L overwrites the lower triangle of each A_i;
+ *             only the lower triangle is referenced.
+ *             'U' (upper): A_i = U^T U, U = L^T overwrites the upper triangle; only the upper
+ *             triangle is referenced (the same factorisation on the transposed view, so the
+ *             results are bit-identical to 'L' on the mirrored storage; SURVEY.md §8(f)
+ *             NEXT-1, LAPACK DPOTRF). Anything else returns -1.
  *  d_n        [batchCount] matrix orders n_i (device).
  *  dA_array   [batchCount] device pointers to the matrices (device array of device ptrs).
  *  d_ldda     [batchCount] leading dimensions (device); must be >= max(1, n_i).
@@ -50,13 +54,13 @@ typedef struct CUstream_st* vb_stream_t; /* == cudaStream_t */
  *               0  success;
  *               k>0 the leading minor of order k is not positive definite: the k-th pivot
  *                  was <= 0 or NaN. Columns 1..k-1 hold L of the leading block; the failing
- *                  pivot value is stored at (k,k); the rest of the lower triangle is
+ *                  pivot value is stored at (k,k); the rest of the referenced triangle is
  *                  implementation-defined (partially updated).
  *              -2  n_i < 0;  -4  ldda_i < max(1,n_i);  -7  n_i > max_n.  (matrix untouched)
  *  batchCount number of matrices (>= 0)                                      (-6 if < 0)
  *  max_n      an upper bound on every n_i (host)                              (-7 if < 0)
  *  stream     CUDA stream.
- * The strict upper triangle and rows n_i..ldda_i-1 are never read nor written.
+ * The other (unreferenced) strict triangle and rows n_i..ldda_i-1 are never read nor written.
  * Matrices must not overlap. Returns 0 / -p / cudaError_t as described above.
  */
 int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,

@@ -32,14 +32,17 @@ cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream) {
 
 cudaError_t ws_free(void* p, cudaStream_t stream) { return cudaFreeAsync(p, stream); }
 
+static bool uplo_ok(char u) { return u == 'L' || u == 'l' || u == 'U' || u == 'u'; }
+
 static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                       int batch, int max_n, bool check_max, cudaStream_t stream) {
-  if (uplo != 'L' && uplo != 'l') return -1;  // 'U' is NEXT-1 (include/vbatched.h)
+  if (!uplo_ok(uplo)) return -1;
+  const bool up = (uplo == 'U' || uplo == 'u');
   if (batch < 0) return -6;
   if (check_max && max_n < 0) return -7;
   if (batch == 0) return 0;
   if (check_max && max_n <= kWarpMaxN)  // all matrices on the warp path: no scan needed
-    return (int)launch_potrf_direct(d_n, dA, d_ldda, d_info, batch, max_n, stream);
+    return (int)launch_potrf_direct(d_n, dA, d_ldda, d_info, batch, max_n, up, stream);
   void* ws = nullptr;
   const size_t bytes = sizeof(Ctrl) + sizeof(int) * (size_t)batch;
   cudaError_t e = ws_alloc(&ws, bytes, stream);
@@ -49,7 +52,8 @@ static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d
   e = launch_scan_bin(d_n, d_ldda, d_info, batch, max_n, check_max, ctrl, order, stream);
   if (e == cudaSuccess) {
     const int hint = check_max ? max_n : (1 << 30);
-    if (hint > 0) e = launch_potrf_paths(d_n, dA, d_ldda, d_info, batch, hint, ctrl, order, stream);
+    if (hint > 0)
+      e = launch_potrf_paths(d_n, dA, d_ldda, d_info, batch, hint, ctrl, order, up, stream);
   }
   cudaError_t e2 = ws_free(ws, stream);
   if (e == cudaSuccess) e = e2;
@@ -80,7 +84,7 @@ size_t vbatched_dpotrf_workspace_size(int batchCount) {
 
 int vbatched_dpotrf_scan(char uplo, const int* d_n, const int* d_ldda, int* d_info, int batchCount,
                          int max_n, void* d_workspace, vb_stream_t stream) {
-  if (uplo != 'L' && uplo != 'l') return -1;
+  if (!uplo_ok(uplo)) return -1;
   if (batchCount < 0) return -5;
   if (max_n < 0) return -6;
   if (batchCount == 0) return 0;
@@ -94,17 +98,18 @@ int vbatched_dpotrf_scan(char uplo, const int* d_n, const int* d_ldda, int* d_in
 int vbatched_dpotrf_factor(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
                            int* d_info, int batchCount, int max_n, void* d_workspace,
                            vb_stream_t stream) {
-  if (uplo != 'L' && uplo != 'l') return -1;
+  if (!uplo_ok(uplo)) return -1;
+  const bool up = (uplo == 'U' || uplo == 'u');
   if (batchCount < 0) return -6;
   if (max_n < 0) return -7;
   if (batchCount == 0) return 0;
   if (!d_workspace) return -8;
   if (max_n <= kWarpMaxN)
-    return (int)launch_potrf_direct(d_n, dA_array, d_ldda, d_info, batchCount, max_n,
+    return (int)launch_potrf_direct(d_n, dA_array, d_ldda, d_info, batchCount, max_n, up,
                                     (cudaStream_t)stream);
   Ctrl* ctrl = static_cast<Ctrl*>(d_workspace);
   return (int)launch_potrf_paths(d_n, dA_array, d_ldda, d_info, batchCount, max_n, ctrl,
-                                 reinterpret_cast<int*>(ctrl + 1), (cudaStream_t)stream);
+                                 reinterpret_cast<int*>(ctrl + 1), up, (cudaStream_t)stream);
 }
 
 int vbatched_dgemm(char transA, char transB, const int* d_m, const int* d_n, const int* d_k,

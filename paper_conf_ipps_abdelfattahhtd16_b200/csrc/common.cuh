@@ -28,7 +28,15 @@ struct Ctrl {
   int pad[6];
 };
 
-constexpr int kWarpMaxN = 32;  // warp-per-matrix path for n <= 32
+constexpr int kWarpMaxN = 32;
+
+// Offset of element (r, c) of the lower factor L (r >= c) in a matrix's storage: uplo 'L' keeps
+// L in the lower triangle, column-major (r + c ld); uplo 'U' keeps U = L^T in the upper
+// triangle, so L(r, c) = U(c, r) sits at c + r ld.
+template <bool UP>
+VB_DEVINL size_t gix(int r, int c, int ld) {
+  return UP ? (size_t)r * ld + c : (size_t)c * ld + r;
+}  // warp-per-matrix path for n <= 32
 
 // FP64 tensor-core MMA: D(8x8) += A(8x4, row) * B(4x8, col). Native SASS: DMMA.8x8x4.
 // Fragment layout (verified on B200 by tools/fp64_peaks.cu): lane l = 4g + q holds
@@ -61,6 +69,11 @@ VB_DEVINL void cp_async8(void* sdst, const void* gsrc, bool pred) {
 VB_DEVINL void cp_async16(void* sdst, const void* gsrc, bool pred) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),
                "r"(pred ? 16 : 0));
+}
+// The barrier tracks this thread's prior cp.async copies (pending count +1 now, the async
+// arrive on completion: zero net arrivals; the phase cannot complete before the copies land).
+VB_DEVINL void cp_async_mbar_arrive(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
 VB_DEVINL void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 template <int N>

@@ -60,7 +60,7 @@ using namespace vb;
 extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA,
                                     const int* h_ldda, int* h_info, int batch, int max_n,
                                     size_t workspace_bytes, vb_stream_t user_stream) {
-  if (uplo != 'L' && uplo != 'l') return -1;
+  if (uplo != 'L' && uplo != 'l' && uplo != 'U' && uplo != 'u') return -1;
   if (batch < 0) return -6;
   if (max_n < 0) return -7;
   if (batch == 0) return 0;
@@ -182,7 +182,7 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
                              cudaMemcpyHostToDevice, sl.stream)) != cudaSuccess) break;
     if ((e = cudaMemcpyAsync(sl.dptr, sl.hptr, sizeof(double*) * (size_t)cnt,
                              cudaMemcpyHostToDevice, sl.stream)) != cudaSuccess) break;
-    int rc = vbatched_dpotrf('L', sl.dmeta, sl.dptr, sl.dmeta + sl.cap, sl.dmeta + 2 * sl.cap, cnt,
+    int rc = vbatched_dpotrf(uplo, sl.dmeta, sl.dptr, sl.dmeta + sl.cap, sl.dmeta + 2 * sl.cap, cnt,
                              cmax, (vb_stream_t)sl.stream);
     if (rc != 0) { e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue; break; }
     for (const Run& r : c.runs)

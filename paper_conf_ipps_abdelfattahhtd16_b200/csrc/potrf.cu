@@ -289,6 +289,7 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
 // pivot). Blocked 16 + 16: POTF2 of columns 0..15 with all 32 rows in registers (which also
 // produces L21), the trailing 16x16 update C22 -= L21 L21^T on DMMA, POTF2 of C22.
 // sv/tv (>= 32 doubles) receive l_cc and 1/l_cc. Returns info.
+template <bool UP>
 VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, int lda,
                             double* ws, double* sv, double* tv) {
   const int nb1 = min(nb, 16), nb2 = nb - nb1;
@@ -304,7 +305,7 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
     for (int c = 0; c < 16; ++c)
       if (c < ncol && lane >= c && lane < nb) {
         T[c * ldt + lane] = a[c];
-        Ag[(size_t)c * lda + lane] = a[c];
+        Ag[gix<UP>(lane, c, lda)] = a[c];
       }
   }
   __syncwarp();
@@ -356,7 +357,7 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
     for (int c = 0; c < 16; ++c)
       if (lane < 16 && c < ncol && r >= c && r < nb2) {
         T22[c * ldt + r] = a[c];
-        A22[(size_t)c * lda + r] = a[c];
+        A22[gix<UP>(r, c, lda)] = a[c];
       }
     info = info2 ? 16 + info2 : 0;
   }
@@ -426,7 +427,7 @@ struct Smem2 {
 // Diagonal 64x64 block by warps 0..3 (named barrier 1): L11 = potf2(C11), inv(L11) -> T12,
 // L21 = C21 inv(L11)^T -> T21, C22 -= L21 L21^T, L22 = potf2(C22), inv(L22) -> T11.
 // Stores L11, L21, L22 (rows < nb) to global (Ad, ld). Sets s.info (1-based, in-block).
-template <class CC>
+template <class CC, bool UP>
 __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int lane, double* Ad,
                                             int ld, bool below) {
   constexpr int LDT = CC::LDT;
@@ -438,7 +439,7 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
   const int nb1 = min(nb, 32), nb2 = nb - nb1;
   DP_START
   if (wg == 0) {
-    const int info = potf2_block32(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
+    const int info = potf2_block32<UP>(T, LDT, nb1, lane, Ad, ld, s.wbuf, s.sv, s.tv);
     DP_MARK(0)
     if (!info && nb2 > 0) trtri32_dmma_warp(T, LDT, s.tv, INV11, LDT, s.S, LDS_T, lane);
     DP_MARK(1)
@@ -460,7 +461,7 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
         for (int h = 0; h < 2; ++h) {
           const int r = 32 + m0 + mt * 8 + g, c = n0 + nt * 8 + 2 * q + h;
           T[c * LDT + r] = acc[mt][nt][h];
-          if (r < nb) Ad[(size_t)c * ld + r] = acc[mt][nt][h];
+          if (r < nb) Ad[gix<UP>(r, c, ld)] = acc[mt][nt][h];
         }
   }
   bar_group(1, 128);
@@ -489,7 +490,7 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
   DP_MARK(4)
   if (wg == 0) {
     double* T22 = T + 32 * LDT + 32;
-    const int info = potf2_block32(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf,
+    const int info = potf2_block32<UP>(T22, LDT, nb2, lane, Ad + (size_t)32 * ld + 32, ld, s.wbuf,
                                    s.sv + 32, s.tv + 32);
     DP_MARK(5)
     if (!info && below) trtri32_dmma_warp(T22, LDT, s.tv + 32, INV22, LDT, s.S, LDS_T, lane);
@@ -501,7 +502,7 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
 }
 
 // Producer (warp 0): chunk kc of the row block at r0 into ring slot gi % STAGES.
-template <class C>
+template <class C, bool UP>
 VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, int n, int ld,
                             int r0, int j0, int lane, bool bulk) {
   const int st = gi % C::STAGES;
@@ -520,13 +521,42 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, i
       const int c = lane - 16;
       bulk_g2s(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * 8, &s.full[st]);
     }
-  } else {  // odd ldda / unaligned base: plain loads by the producer warp, then arrive
-    const int ra = min(C::MB, n - r0), rb = min(C::NB, n - j0);
-    for (int c = 0; c < C::KC; ++c) {
-      const double* col = A + (size_t)(k0 + c) * ld;
-      for (int r = lane; r < ra; r += 32) s.a[st][c][r] = col[r0 + r];
-      for (int r = lane; r < rb; r += 32) s.b[st][c][r] = col[j0 + r];
+  } else {
+    // Odd ldda / unaligned base ('L'), or uplo 'U': the chunk is gathered with 8-byte cp.async
+    // (LDGSTS, no register staging; rows >= n are zero-filled). 'L': lanes run down a column;
+    // 'U': L's rows are contiguous in storage (16 k-values of one row = 128 B), 16 lanes per
+    // row. Every lane's copies are tracked by the full barrier (cp.async.mbarrier.arrive: zero
+    // net arrivals) and lane 0 adds the one expected arrival.
+    static_assert(C::KC == 16 && C::MB % 32 == 0 && C::NB % 32 == 0, "copy shapes");
+    if (UP) {
+      const int c = lane & 15;
+#pragma unroll 4
+      for (int r = lane >> 4; r < C::MB; r += 2) {
+        const bool p = r0 + r < n;
+        cp_async8(&s.a[st][c][r], A + (p ? (size_t)(r0 + r) * ld + k0 + c : 0), p);
+      }
+#pragma unroll 4
+      for (int r = lane >> 4; r < C::NB; r += 2) {
+        const bool p = j0 + r < n;
+        cp_async8(&s.b[st][c][r], A + (p ? (size_t)(j0 + r) * ld + k0 + c : 0), p);
+      }
+    } else {
+#pragma unroll 4
+      for (int c = 0; c < C::KC; ++c) {
+        const double* col = A + (size_t)(k0 + c) * ld;
+#pragma unroll
+        for (int r = lane; r < C::MB; r += 32) {
+          const bool p = r0 + r < n;
+          cp_async8(&s.a[st][c][r], p ? col + r0 + r : A, p);
+        }
+#pragma unroll
+        for (int r = lane; r < C::NB; r += 32) {
+          const bool p = j0 + r < n;
+          cp_async8(&s.b[st][c][r], p ? col + j0 + r : A, p);
+        }
+      }
     }
+    cp_async_mbar_arrive(&s.full[st]);
     __syncwarp();
     if (lane == 0) mbar_arrive(&s.full[st]);
   }
@@ -614,11 +644,11 @@ VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
 // panel_done mbarrier for panel p-1 (the consumers arrive after storing and fencing that
 // panel's L), so TMA never reads a column before it is final.
 
-template <class C>
+template <class C, bool UP>
 VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int lane,
                                uint32_t& gchunk, uint32_t& gpanel) {
   constexpr int NB = C::NB, MB = C::MB, KC = C::KC;
-  const bool bulk = ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
+  const bool bulk = !UP && ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
   const int npan = (n + NB - 1) / NB;
   int done = npan;  // panels the consumers will complete for this matrix
   fence_proxy_async();
@@ -632,7 +662,7 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
       const int rn = (min(MB, n - j0) + 1) & ~1;
       bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + j0, rn * 8);
     }
-    for (int kc = 0; kc < nk_free; ++kc) issue_chunk2<C>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
+    for (int kc = 0; kc < nk_free; ++kc) issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
     if (lane == 0) mbar_wait(&s.panel_done, (gpanel + p - 1) & 1);  // panel p-1 is stored
     __syncwarp();
     if (s.info) {  // the consumers failed in panel p-1 and stop there (they also drain the
@@ -645,7 +675,7 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
         bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * 8);
       }
       for (int kc = (r0 == j0 ? nk_free : 0); kc < nk; ++kc)
-        issue_chunk2<C>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
+        issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
     }
   }
   gpanel += done;
@@ -685,7 +715,7 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
   }
 }
 
-template <class C>
+template <class C, bool UP>
 VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int ld,
                                int* info_out, uint32_t& gchunk, uint32_t& gpanel) {
   constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
@@ -719,7 +749,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
           for (int h = 0; h < 2; ++h) {
             const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
             const bool v = row < n && col < j0 + nb && row >= col;
-            acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+            acc[mt][nt][h] = v ? __ldcg(A + gix<UP>(row, col, ld)) : 0.0;
           }
       VB_T0(t_k)
       // In a panel's first row block the diagonal-block warps only need the column tiles on
@@ -750,7 +780,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
               s.T[nt * 8 + 2 * q + 1][wrow + mt * 8 + g] = acc[mt][nt][1];
             }
           bar_group(2, CT);
-          diag_block64v2(s, nb, warp, lane, A + (size_t)j0 * ld + j0, ld, below);
+          diag_block64v2<C, UP>(s, nb, warp, lane, A + (size_t)j0 * ld + j0, ld, below);
           bar_group(3, CT);
           failed = s.info != 0;
         } else {
@@ -767,7 +797,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
                 for (int h = 0; h < 2; ++h) {
                   const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
                   if (row < n && row >= j0 + nb && col < nb)
-                    A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+                    A[gix<UP>(row, j0 + col, ld)] = acc[mt][nt][h];
                 }
           }
         }
@@ -785,7 +815,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
               const int row = r0 + wrow + mt * 8 + g, col = nt * 8 + 2 * q + h;
-              if (row < n && col < nb) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+              if (row < n && col < nb) A[gix<UP>(row, j0 + col, ld)] = acc[mt][nt][h];
             }
       }
       VB_ADD(2, t_t)
@@ -813,7 +843,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
   gpanel += npan_done;
 }
 
-template <class C>
+template <class C, bool UP>
 __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     potrf_blocked3_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                           const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -848,10 +878,10 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     const int m = order[start + it];
     TL_BEGIN(t_tl)
     if (warp == kV3Consumers) {
-      produce_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
+      produce_matrix3<C, UP>(s, dA[m], d_n[m], d_ldda[m], lane, gchunk, gpanel);
     } else {
       VB_T0(t_m)
-      consume_matrix3<C>(s, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gpanel);
+      consume_matrix3<C, UP>(s, dA[m], d_n[m], d_ldda[m], d_info + m, gchunk, gpanel);
       VB_ADD(4, t_m)
     }
     TL_END(tid == 0, t_tl, m, 30)
@@ -879,6 +909,7 @@ struct SmallSmem {
 };
 
 // acc (32 x 32 block at rows r0.., cols j0..) = A - L[r0:, 0:j0] L[j0:j0+32, 0:j0]^T
+template <bool UP>
 VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restrict__ A, int n,
                                   int ld, int r0, int j0, int nb, bool diag, int lane) {
   const int g = lane >> 2, q = lane & 3;
@@ -890,7 +921,7 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restri
       for (int h = 0; h < 2; ++h) {
         const int row = r0 + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
         const bool v = row < n && col < j0 + nb && (!diag || row >= col);
-        acc[mt][nt][h] = v ? __ldcg(A + (size_t)col * ld + row) : 0.0;
+        acc[mt][nt][h] = v ? __ldcg(A + gix<UP>(row, col, ld)) : 0.0;
       }
   bool rv[4], cv[4];
 #pragma unroll
@@ -900,12 +931,11 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restri
   }
 #pragma unroll 2
   for (int k = q; k < j0; k += 4) {
-    const double* col = A + (size_t)k * ld;
     double fa[4], fb[4];
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
-      fa[t] = rv[t] ? -__ldcg(col + r0 + t * 8 + g) : 0.0;
-      fb[t] = cv[t] ? __ldcg(col + j0 + t * 8 + g) : 0.0;
+      fa[t] = rv[t] ? -__ldcg(A + gix<UP>(r0 + t * 8 + g, k, ld)) : 0.0;
+      fb[t] = cv[t] ? __ldcg(A + gix<UP>(j0 + t * 8 + g, k, ld)) : 0.0;
     }
 #pragma unroll
     for (int mt = 0; mt < 4; ++mt)
@@ -916,6 +946,7 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restri
 
 // X = C inv(L11)^T for a 32 x 32 block in registers (inv[k][n] upper in k,n: zero blocks
 // skipped), then direct stores of rows < n.
+template <bool UP>
 VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], double* __restrict__ A,
                                 int n, int ld, int r0, int j0, int lane) {
   const int g = lane >> 2, q = lane & 3;
@@ -945,10 +976,11 @@ VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], double* __
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
-        if (row < n) A[(size_t)(j0 + col) * ld + row] = x[mt][nt][h];
+        if (row < n) A[gix<UP>(row, j0 + col, ld)] = x[mt][nt][h];
       }
 }
 
+template <bool UP>
 __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     potrf_small_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                        const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -980,7 +1012,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
         const int r0 = j0 + 32 * b;
         double acc[4][4][2];
         VB_T0(t_g)
-        small_panel_update(acc, A, n, ld, r0, j0, nb, b == 0, lane);
+        small_panel_update<UP>(acc, A, n, ld, r0, j0, nb, b == 0, lane);
         VB_ADD(0, t_g)
         if (b == 0) {  // warp 0: the diagonal block
           const int g = lane >> 2, q = lane & 3;
@@ -993,7 +1025,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
             }
           __syncwarp();
           VB_T0(t_p)
-          const int info = potf2_block32(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
+          const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
                                          s.wbuf, s.sv, s.tv);
           VB_ADD(1, t_p)
           VB_T0(t_i)
@@ -1009,7 +1041,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
             failed = s.info != 0;
           }
           VB_T0(t_s)
-          if (!failed) small_trsm_store(s, acc, A, n, ld, r0, j0, lane);
+          if (!failed) small_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
           VB_ADD(3, t_s)
         }
         if (failed) break;
@@ -1065,6 +1097,7 @@ VB_DEVINL void inv8_blocks(WSmem& s, int lane) {
 
 // In-register TRSM of a 32 x 32 C block (C-fragment layout) against L11 by 8-column block
 // substitution; result stored to global rows < n.
+template <bool UP>
 VB_DEVINL void wsmall_trsm_store(WSmem& s, double (&acc)[4][4][2], double* __restrict__ A, int n,
                                  int ld, int r0, int j0, int lane) {
   const int g = lane >> 2, q = lane & 3;
@@ -1109,10 +1142,11 @@ VB_DEVINL void wsmall_trsm_store(WSmem& s, double (&acc)[4][4][2], double* __res
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
-        if (row < n) A[(size_t)(j0 + col) * ld + row] = acc[mt][nt][h];
+        if (row < n) A[gix<UP>(row, j0 + col, ld)] = acc[mt][nt][h];
       }
 }
 
+template <bool UP>
 __global__ void __launch_bounds__(32, 16)
     potrf_wsmall_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                         const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -1140,7 +1174,7 @@ __global__ void __launch_bounds__(32, 16)
       for (int b = 0; b < nblk; ++b) {
         const int r0 = j0 + 32 * b;
         double acc[4][4][2];
-        small_panel_update(acc, A, n, ld, r0, j0, nb, b == 0, lane);
+        small_panel_update<UP>(acc, A, n, ld, r0, j0, nb, b == 0, lane);
         if (b == 0) {
           const int g = lane >> 2, q = lane & 3;
 #pragma unroll
@@ -1151,12 +1185,12 @@ __global__ void __launch_bounds__(32, 16)
               s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
             }
           __syncwarp();
-          info = potf2_block32(&s.T[0][0], LDW, nb, lane, A + (size_t)j0 * ld + j0, ld, s.wbuf,
+          info = potf2_block32<UP>(&s.T[0][0], LDW, nb, lane, A + (size_t)j0 * ld + j0, ld, s.wbuf,
                                s.sv, s.tv);
           if (info) break;
           if (nblk > 1) inv8_blocks(s, lane);
         } else {
-          wsmall_trsm_store(s, acc, A, n, ld, r0, j0, lane);
+          wsmall_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
         }
       }
       if (info) {
@@ -1178,18 +1212,18 @@ struct WarpSmem {
 };
 
 // One matrix (n <= NM) by one warp, rows in registers: one HBM read, one HBM write.
-template <int NM>
+template <int NM, bool UP>
 VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* info_out, int lane,
                                  double* ws, double* sv, double* tv) {
   double a[NM];
 #pragma unroll
   for (int c = 0; c < NM; ++c)
-    a[c] = (c < n && lane >= c && lane < n) ? A[(size_t)c * ld + lane] : selp(c == lane, 1.0, 0.0);
+    a[c] = (c < n && lane >= c && lane < n) ? A[gix<UP>(lane, c, ld)] : selp(c == lane, 1.0, 0.0);
   const int info = potf2_regs_warp<NM>(a, n, lane, ws, sv, tv);
   const int ncol = info ? info : n;
 #pragma unroll
   for (int c = 0; c < NM; ++c)
-    if (c < ncol && lane >= c && lane < n) A[(size_t)c * ld + lane] = a[c];
+    if (c < ncol && lane >= c && lane < n) A[gix<UP>(lane, c, ld)] = a[c];
   if (lane == 0 && info) *info_out = info;
   __syncwarp();
 }
@@ -1198,6 +1232,7 @@ VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* inf
 // wait_upstream: 1 when launched directly after the scan (the only factorisation kernel),
 // 0 when launched after a blocked kernel (whose CTAs passed the scan's completion before
 // releasing this grid, so the scan's outputs are already visible).
+template <bool UP>
 __global__ void __launch_bounds__(32 * kWarpsPerCta)
     potrf_warp_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                       const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -1218,11 +1253,11 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
     const int n = d_n[m], ld = d_ldda[m];
     TL_BEGIN(t_tl)
     if (n <= 8)
-      potrf_warp_matrix<8>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<8, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else if (n <= 16)
-      potrf_warp_matrix<16>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<16, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else
-      potrf_warp_matrix<32>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<32, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     TL_END(lane == 0, t_tl, m, 40)
   }
 }
@@ -1230,6 +1265,7 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 // Direct warp path for batches whose max_n <= 32 (no scan, no sort: with every matrix this
 // small there is nothing to balance): warp w validates (info -2/-4/-7, as the scan would) and
 // factors matrices w, w + nwarps, ... One launch per call — the latency path for C1.
+template <bool UP>
 __global__ void __launch_bounds__(32 * kWarpsPerCta)
     potrf_warp_direct_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
                              const int* __restrict__ d_ldda, int* __restrict__ d_info, int batch,
@@ -1246,11 +1282,11 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
     if (lane == 0) d_info[m] = code;
     if (code != 0 || n == 0) continue;
     if (n <= 8)
-      potrf_warp_matrix<8>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<8, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else if (n <= 16)
-      potrf_warp_matrix<16>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<16, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else
-      potrf_warp_matrix<32>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<32, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
   }
 }
 
@@ -1281,18 +1317,22 @@ static cudaError_t init_device_info() {
   int sms = 0;
   e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d>,
+  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d, false>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64d>));
   if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64, potrf_blocked3_kernel<Cfg64d>,
+  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64d>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64, potrf_blocked3_kernel<Cfg64d, false>,
                                                     32 * (Cfg64d::WARPS + 1), sizeof(Smem2<Cfg64d>));
   if (e != cudaSuccess) return e;
   if (g_occ64 < 1) g_occ64 = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_kernel,
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_kernel<false>,
                                                     32 * kSmallWarps, 0);
   if (e != cudaSuccess) return e;
   if (g_occ_small < 1) g_occ_small = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_wsmall, potrf_wsmall_kernel, 32, 0);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_wsmall, potrf_wsmall_kernel<false>, 32,
+                                                    0);
   if (e != cudaSuccess) return e;
   if (g_occ_wsmall < 1) g_occ_wsmall = 1;
   {
@@ -1309,7 +1349,7 @@ static cudaError_t init_device_info() {
 // the previous kernel frees at its tail).
 cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
-                               cudaStream_t stream) {
+                               bool up, cudaStream_t stream) {
   cudaError_t e = init_device_info();
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -1324,8 +1364,9 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
     cfg.blockDim = dim3(32 * (Cfg64d::WARPS + 1));
     cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
     cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64d>);
-    e = cudaLaunchKernelEx(&cfg, potrf_blocked3_kernel<Cfg64d>, d_n, dA, d_ldda, d_info, ctrl,
-                           order, 0, wait);
+    e = cudaLaunchKernelEx(&cfg, up ? potrf_blocked3_kernel<Cfg64d, true>
+                                    : potrf_blocked3_kernel<Cfg64d, false>,
+                           d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
@@ -1334,14 +1375,14 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
       cfg.blockDim = dim3(32 * kSmallWarps);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
       cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, potrf_small_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 1,
-                             wait);
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true> : potrf_small_kernel<false>, d_n,
+                             dA, d_ldda, d_info, ctrl, order, 1, wait);
     } else {
       cfg.blockDim = dim3(32);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
       cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, potrf_wsmall_kernel, d_n, dA, d_ldda, d_info, ctrl, order, 1,
-                             wait);
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_wsmall_kernel<true> : potrf_wsmall_kernel<false>, d_n,
+                             dA, d_ldda, d_info, ctrl, order, 1, wait);
     }
     if (e != cudaSuccess) return e;
     wait = 0;
@@ -1351,7 +1392,8 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.gridDim = dim3(std::max(1, std::min((warps + kWarpsPerCta - 1) / kWarpsPerCta,
                                           g_num_sms * 8)));
   cfg.dynamicSmemBytes = 0;
-  return cudaLaunchKernelEx(&cfg, potrf_warp_kernel, d_n, dA, d_ldda, d_info, ctrl, order, wait);
+  return cudaLaunchKernelEx(&cfg, up ? potrf_warp_kernel<true> : potrf_warp_kernel<false>, d_n, dA,
+                            d_ldda, d_info, ctrl, order, wait);
 }
 
 void potrf_occupancy(int* out4) {
@@ -1369,12 +1411,16 @@ int potrf_num_launches(int max_n_hint) {
 }
 
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
-                                int batch, int max_n, cudaStream_t stream) {
+                                int batch, int max_n, bool up, cudaStream_t stream) {
   cudaError_t e = init_device_info();
   if (e != cudaSuccess) return e;
   const int grid = std::max(1, std::min((batch + kWarpsPerCta - 1) / kWarpsPerCta, g_num_sms * 16));
-  potrf_warp_direct_kernel<<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info, batch,
-                                                                   max_n);
+  if (up)
+    potrf_warp_direct_kernel<true><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info,
+                                                                          batch, max_n);
+  else
+    potrf_warp_direct_kernel<false><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info,
+                                                                           batch, max_n);
   return cudaGetLastError();
 }
 

@@ -37,7 +37,8 @@ def test_version_string():
 def test_host_argument_checks_without_gpu():
     # host scalars are checked before any CUDA call (include/vbatched.h conventions)
     assert vb.vbatched_dpotrf("X", 0, 0, 0, 0, 1, 4, stream=0, check=False) == -1
-    assert vb.vbatched_dpotrf("U", 0, 0, 0, 0, 1, 4, stream=0, check=False) == -1
+    assert vb.vbatched_dpotrf("u", 0, 0, 0, 0, -1, 4, stream=0, check=False) == -6  # 'U' accepted
+    assert vb.vbatched_dpotrf("U", 0, 0, 0, 0, 0, 4, stream=0, check=False) == 0
     assert vb.vbatched_dpotrf("L", 0, 0, 0, 0, -1, 4, stream=0, check=False) == -6
     assert vb.vbatched_dpotrf("L", 0, 0, 0, 0, 1, -3, stream=0, check=False) == -7
     assert vb.vbatched_dpotrf("L", 0, 0, 0, 0, 0, 0, stream=0, check=False) == 0
@@ -58,7 +59,7 @@ def test_host_api_argument_checks_and_codes():
     info = np.zeros(4, dtype=np.int32)
     ptrs = np.zeros(4, dtype=np.int64)
     assert vb.vbatched_dpotrf_host("L", n, ptrs, ld, info, 4, -1, check=False) == -7
-    assert vb.vbatched_dpotrf_host("U", n, ptrs, ld, info, 4, 8, check=False) == -1
+    assert vb.vbatched_dpotrf_host("Q", n, ptrs, ld, info, 4, 8, check=False) == -1
 
 
 def test_kernel_launch_count():

@@ -328,7 +328,7 @@ def test_argument_errors_and_empty():
     from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
     db = DeviceBatch(np.array([4], dtype=np.int32)).fill()
     assert vbatched_dpotrf("X", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, 4, check=False) == -1
-    assert vbatched_dpotrf("U", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, 4, check=False) == -1
+    assert vbatched_dpotrf("X", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, 4, check=False) == -1
     assert vbatched_dpotrf("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, -1, 4, check=False) == -6
     assert vbatched_dpotrf("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, 1, -1, check=False) == -7
     assert vbatched_dpotrf("L", 0, 0, 0, 0, 0, 0, check=False) == 0
@@ -388,3 +388,66 @@ def test_repeat_bit_identical(cfg):
             ref, ref_info = out, info
             continue
         assert torch.equal(out, ref) and np.array_equal(info, ref_info)
+
+
+@pytest.mark.parametrize("ldda_mode", ["pad32", "tight"])
+def test_uplo_upper_matches_lower_bitwise(ldda_mode):
+    """uplo='U' (LAPACK DPOTRF): A = U^T U with only the upper triangle
+    referenced. The kernels run the same arithmetic on the transposed view, so U^T must equal
+    the 'L' run's factor bit for bit (info too); the strict lower triangle and the padding rows
+    stay untouched (NaN poison), and the factor passes the oracle gates."""
+    sizes = [1, 2, 7, 16, 31, 32, 33, 40, 64, 65, 96, 127, 128, 129, 160, 192, 255, 256, 257,
+             300, 384, 511, 513, 640, 700, 1024]
+    fail = {3: 5, 10: 60, 17: 200, 21: 129, 24: 650}  # slot -> failing pivot (1-based)
+    n = np.array(sizes, dtype=np.int32)
+    dl = DeviceBatch(n, seed=21, ldda_mode=ldda_mode)
+    du = DeviceBatch(n, seed=21, ldda_mode=ldda_mode)
+    inputs = {}
+    for i, ni in enumerate(sizes):
+        A = vbgen.f1_matrix(21, i, ni)
+        if i in fail:
+            k = fail[i]
+            A[k - 1, k - 1] = -A[k - 1, k - 1]
+        inputs[i] = A
+        dl.set_matrix(i, A, uplo="L")
+        du.set_matrix(i, A, uplo="U")
+    dl.dpotrf(uplo="L")
+    du.dpotrf(uplo="U")
+    torch.cuda.synchronize()
+    il, iu = dl.info(), du.info()
+    assert list(il) == list(iu) == [fail.get(i, 0) for i in range(len(sizes))]
+    for i, ni in enumerate(sizes):
+        bl, bu = dl.block(i), du.block(i)
+        k = ni if il[i] == 0 else il[i] - 1  # defined leading block
+        low = np.tril(np.ones((k, k), bool))
+        Lb = bl[:k, :k].view(np.uint64)
+        Ub = bu[:k, :k].T.view(np.uint64)
+        assert np.array_equal(Lb[low], Ub[low]), i
+        # strict lower triangle and padding rows of the 'U' storage: never touched
+        strict_low = np.tril(np.ones((ni, ni), bool), -1)
+        assert np.all(bu[:ni, :ni].view(np.uint64)[strict_low] == POISON), i
+        if bu.shape[0] > ni:
+            assert np.all(bu[ni:, :].view(np.uint64) == POISON), i
+        r = compare_with_oracle(inputs[i], bu[:ni, :ni].T.copy(), iu[i])
+        assert r["ok"], (i, r)
+
+
+def test_uplo_upper_device_generated_c3_sample():
+    """uplo='U' on device-generated upper storage (vbgen poison bit 1): the first 600 matrices of
+    C3 with 5 % non-SPD; info and U^T bitwise equal to the 'L' run, lower triangle untouched."""
+    n = vbgen.sizes("C3")[:600]
+    dl = DeviceBatch(n, seed=3, nonspd_mod=20).fill(poison=True)
+    du = DeviceBatch(n, seed=3, nonspd_mod=20).fill(poison=True, uplo="U")
+    dl.dpotrf(uplo="L")
+    du.dpotrf(uplo="U")
+    torch.cuda.synchronize()
+    il, iu = dl.info(), du.info()
+    assert np.array_equal(il, iu) and (il > 0).sum() == 30
+    for i in range(0, 600, 7):
+        ni = int(n[i])
+        k = ni if il[i] == 0 else il[i] - 1
+        low = np.tril(np.ones((k, k), bool))
+        bl, bu = dl.block(i), du.block(i)
+        assert np.array_equal(bl[:k, :k].view(np.uint64)[low], bu[:k, :k].T.view(np.uint64)[low]), i
+        strict_low = np.tril(np.ones((ni, ni), bool), -1)
+        assert np.all(bu[:ni, :ni].view(np.uint64)[strict_low] == POISON), i

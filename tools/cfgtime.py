@@ -12,6 +12,7 @@ from harness import DeviceBatch  # noqa: E402
 
 reps = int(os.environ.get("REPS", "5"))
 tag = os.environ.get("TAG", "")
+uplo = os.environ.get("UPLO", "L")
 for cfg in sys.argv[1:]:
     if cfg.startswith("u"):
         nn, cnt = (int(x) for x in cfg[1:].split("x"))
@@ -22,11 +23,11 @@ for cfg in sys.argv[1:]:
     db = DeviceBatch(n, seed=seed, nonspd_mod=mod)
     ts = []
     for it in range(reps + 1):
-        db.fill()
+        db.fill(uplo=uplo)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        db.dpotrf()
+        db.dpotrf(uplo=uplo)
         e1.record()
         torch.cuda.synchronize()
         if it:

@@ -24,8 +24,9 @@ def lib():
 
 
 def fill_f1(seed: int, batch: int, d_n: int, d_ldda: int, d_ptrs: int, d_gidx: int | None,
-            nonspd_mod: int, poison: bool, stream: int) -> None:
+            nonspd_mod: int, poison: int, stream: int) -> None:
+    """poison: bit 0 = NaN sentinels outside the referenced triangle, bit 1 = upper storage."""
     rc = lib().vbgen_fill_f1(int(seed), int(batch), d_n, d_ldda, d_ptrs, d_gidx, int(nonspd_mod),
-                             1 if poison else 0, stream)
+                             int(poison), stream)
     if rc != 0:
         raise RuntimeError(f"vbgen_fill_f1 failed: cudaError {rc}")

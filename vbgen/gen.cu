@@ -7,8 +7,10 @@
 //                     double* const* d_A, const int* d_gidx, int nonspd_mod, int poison,
 //                     cudaStream_t stream)
 //     d_n/d_ldda/d_A/d_gidx: device arrays of length batch (d_gidx may be NULL -> gidx = i).
-//     Writes the lower triangle (and, if poison != 0, NaN-payload sentinels into the strict
-//     upper triangle and the padding rows n..ldda-1). Returns a cudaError_t.
+//     Writes the lower triangle (and, if poison bit 0 is set, NaN-payload sentinels into the
+//     strict upper triangle and the padding rows n..ldda-1). Poison bit 1 selects upper
+//     storage instead (the same symmetric matrix in the upper triangle, for uplo 'U'; the
+//     sentinels then go to the strict lower triangle). Returns a cudaError_t.
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -37,13 +39,16 @@ __global__ void fill_f1_kernel(uint64_t seed, int batch, const int* __restrict__
     int kneg = -1;
     if (nonspd_mod > 0 && (int)(g % (uint64_t)nonspd_mod) == nonspd_mod - 1)
       kneg = (int)(splitmix64(s0 ^ g ^ 0x5EEDull) % (uint64_t)n);
-    const int rows = poison ? ld : n;
+    const bool up = (poison & 2) != 0, poi = (poison & 1) != 0;
+    const int rows = poi ? ld : n;
     for (int j = 0; j < n; ++j) {
       double* col = A + (size_t)j * ld;
-      for (int i = (poison ? 0 : j) + threadIdx.x; i < rows; i += blockDim.x) {
+      const int i0 = (poi || up) ? 0 : j, i1 = (up && !poi) ? j + 1 : rows;
+      for (int i = i0 + threadIdx.x; i < i1; i += blockDim.x) {
         double v;
-        if (i >= j && i < n) {
-          const uint64_t key = (g << 42) ^ ((uint64_t)i << 21) ^ (uint64_t)j;
+        if (up ? (i <= j) : (i >= j && i < n)) {
+          const int r = i > j ? i : j, c = i > j ? j : i;
+          const uint64_t key = (g << 42) ^ ((uint64_t)r << 21) ^ (uint64_t)c;
           v = (double)(splitmix64(s0 ^ key) >> 11) * 0x1.0p-53;
           if (i == j) {
             v = v + (double)n;
