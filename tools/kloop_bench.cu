@@ -129,13 +129,13 @@ int main() {
   CK(cudaMalloc(&base, sizeof(double) * (size_t)nmat * n * n)); CK(cudaMalloc(&sink, 64));
   CK(cudaMemset(base, 0, sizeof(double) * (size_t)nmat * n * n));
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-  for (int K : {256}) {
-    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms, 2);
-    run<64, 16, 3, 8, 1>(base, nmat, n, K, sink, sms, 1);
-    run<64, 16, 3, 8, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
-    run<64, 16, 4, 8, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
+  for (int K : {256, 512}) {
     run<64, 16, 3, 8, 1, 128, 2, 1>(base, nmat, n, K, sink, sms, 2);
-    run<64, 16, 3, 16, 1, 128, 1, 1>(base, nmat, n, K, sink, sms, 1);
+    // the production shape: MB = 64 (4 consumer warps) + producer, 3 CTAs per SM
+    run<64, 16, 2, 4, 1, 64, 3, 1>(base, nmat, n, K, sink, sms, 3);
+    run<64, 16, 3, 4, 1, 64, 3, 1>(base, nmat, n, K, sink, sms, 3);
+    run<64, 16, 4, 4, 1, 64, 3, 1>(base, nmat, n, K, sink, sms, 3);
+    run<64, 16, 2, 4, 1, 64, 4, 1>(base, nmat, n, K, sink, sms, 4);
   }
   return 0;
 }
