@@ -136,11 +136,34 @@ int vbatched_dsyrk(char uplo, char trans, const int* d_n, const int* d_k, double
  *   diag 'N' or 'U' (unit). Cholesky uses side 'R', uplo 'L', transA 'T', diag 'N'
  *   ("C2 = C2 C1^-T"). Implemented as an in-shared-memory inversion of the
  *   diagonal blocks (TRTRI) followed by DMMA GEMMs, the design PAPER.md:760-772 describes.
- *   Supported now: side 'R' with any uplo/transA/diag; side 'L' returns -1 (NEXT-2). */
+ *   Every side/uplo/transA/diag combination (side 'L' runs the side-'R' kernel on the
+ *   transposed view: op(A) X = alpha B <=> X^T op(A)^T = alpha B^T).
+ *   A is m_i x m_i for side 'L', n_i x n_i for side 'R'. Bad side -1, uplo -2, transA -3,
+ *   diag -4. */
 int vbatched_dtrsm(char side, char uplo, char transA, char diag, const int* d_m, const int* d_n,
                    double alpha, const double* const* dA_array, const int* d_ldda,
                    double* const* dB_array, const int* d_lddb, int batchCount, int max_m,
                    int max_n, vb_stream_t stream);
+
+/* vbatched_dpotrs — solve A_i X_i = B_i with the factor vbatched_dpotrf left in dA_array
+ * (the paper's "factorization and solve routines", PAPER.md:183-185;
+ * LAPACK DPOTRS). uplo as passed to vbatched_dpotrf: 'L' solves L Y = B then L^T X = Y,
+ * 'U' solves U^T Y = B then U X = Y — two vbatched_dtrsm (side 'L') launches.
+ *  d_n, d_nrhs  [batchCount] orders n_i and right-hand-side counts nrhs_i (device);
+ *  dB_array     B_i: n_i x nrhs_i, column-major, leading dimension d_lddb[i] >= max(1,n_i);
+ *               overwritten by X_i. A_i is only read (its referenced triangle).
+ *  max_n, max_nrhs: host upper bounds. Returns uplo -1, batchCount -8, max_n -9,
+ *  max_nrhs -10 (host scalars), 0 or a cudaError_t. No per-matrix info (as DPOTRS). */
+int vbatched_dpotrs(char uplo, const int* d_n, const int* d_nrhs, const double* const* dA_array,
+                    const int* d_ldda, double* const* dB_array, const int* d_lddb,
+                    int batchCount, int max_n, int max_nrhs, vb_stream_t stream);
+
+/* vbatched_dposv — vbatched_dpotrf followed by vbatched_dpotrs (LAPACK DPOSV): A_i is
+ * overwritten by its factor, B_i by X_i; d_info as vbatched_dpotrf, and a matrix with
+ * info != 0 keeps B_i unchanged. Returns uplo -1, batchCount -9, max_n -10, max_nrhs -11. */
+int vbatched_dposv(char uplo, const int* d_n, const int* d_nrhs, double* const* dA_array,
+                   const int* d_ldda, double* const* dB_array, const int* d_lddb, int* d_info,
+                   int batchCount, int max_n, int max_nrhs, vb_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------
  * Host helpers (pure host, deterministic, no CUDA).

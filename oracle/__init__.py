@@ -140,6 +140,32 @@ def dtrsm(side, uplo, transA, diag, alpha, A, B):
     return B
 
 
+def dpotrs(uplo, F, B):
+    """Solve A X = B from the Cholesky factor F of A, step by step as LAPACK DPOTRS defines it
+    (SURVEY.md §8(f) NEXT-4): 'L' (F = L, A = L L^T): L Y = B, then L^T X = Y; 'U' (F = U,
+    A = U^T U): U^T Y = B, then U X = Y. Each step is the oracle's plain triangular solve."""
+    if uplo == "L":
+        Y = dtrsm("L", "L", "N", "N", 1.0, F, B)
+        return dtrsm("L", "L", "T", "N", 1.0, F, Y)
+    Y = dtrsm("L", "U", "T", "N", 1.0, F, B)
+    return dtrsm("L", "U", "N", "N", 1.0, F, Y)
+
+
+def dposv(uplo, A, B):
+    """LAPACK DPOSV: factor A (the oracle's unblocked Cholesky of the referenced triangle), then
+    dpotrs; on info != 0 B is returned unchanged. Returns (X, F, info)."""
+    A = np.asarray(A, dtype=np.float64)
+    if uplo == "L":
+        L, info = dpotrf(np.asfortranarray(A))
+        F = np.tril(L)
+    else:
+        L, info = dpotrf(np.asfortranarray(A.T))  # U = L^T of the transposed (mirrored) view
+        F = np.triu(L.T)
+    if info != 0:
+        return np.array(B, dtype=np.float64, copy=True), F, info
+    return dpotrs(uplo, F, B), F, info
+
+
 def backward_error(A0: np.ndarray, L: np.ndarray, info: int) -> float:
     """||A - L L^T||_F / (nb ||A||_F eps), eps = 2^-53, long double (SURVEY §8(c) #13)."""
     A0 = np.asfortranarray(A0, dtype=np.float64)

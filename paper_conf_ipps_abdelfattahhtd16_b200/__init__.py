@@ -57,6 +57,8 @@ def lib() -> ctypes.CDLL:
         L.vbatched_dsyrk.argtypes = [_c, _c, _vp, _vp, _d, _vp, _vp, _d, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_dtrsm.argtypes = [_c, _c, _c, _c, _vp, _vp, _d, _vp, _vp, _vp, _vp, _i, _i, _i,
                                      _vp]
+        L.vbatched_dpotrs.argtypes = [_c, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
+        L.vbatched_dposv.argtypes = [_c, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_partition_lpt.argtypes = [_vp, _i, _i, _vp]
         L.vbatched_version.restype = ctypes.c_char_p
         L.vbatched_dpotrf_kernel_launches.argtypes = [_i]
@@ -67,6 +69,7 @@ def lib() -> ctypes.CDLL:
         for name in ("vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
                      "vbatched_dpotrf_scan", "vbatched_dpotrf_factor",
                      "vbatched_dgemm", "vbatched_dsyrk", "vbatched_dtrsm",
+                     "vbatched_dpotrs", "vbatched_dposv",
                      "vbatched_partition_lpt", "vbatched_host_free"):
             getattr(L, name).restype = _i
         _lib = L
@@ -168,6 +171,22 @@ def vbatched_dtrsm(side, uplo, transA, diag, m, n, alpha, dA_array, ldda, dB_arr
                               float(alpha), _ptr(dA_array), _ptr(ldda), _ptr(dB_array), _ptr(lddb),
                               int(batchCount), int(max_m), int(max_n), _stream(stream))
     return _check(rc, "vbatched_dtrsm") if check else rc
+
+
+def vbatched_dpotrs(uplo, n, nrhs, dA_array, ldda, dB_array, lddb, batchCount, max_n, max_nrhs,
+                    stream=None, check=True):
+    rc = lib().vbatched_dpotrs(_ch(uplo), _ptr(n), _ptr(nrhs), _ptr(dA_array), _ptr(ldda),
+                               _ptr(dB_array), _ptr(lddb), int(batchCount), int(max_n),
+                               int(max_nrhs), _stream(stream))
+    return _check(rc, "vbatched_dpotrs") if check else rc
+
+
+def vbatched_dposv(uplo, n, nrhs, dA_array, ldda, dB_array, lddb, info, batchCount, max_n,
+                   max_nrhs, stream=None, check=True):
+    rc = lib().vbatched_dposv(_ch(uplo), _ptr(n), _ptr(nrhs), _ptr(dA_array), _ptr(ldda),
+                              _ptr(dB_array), _ptr(lddb), _ptr(info), int(batchCount), int(max_n),
+                              int(max_nrhs), _stream(stream))
+    return _check(rc, "vbatched_dposv") if check else rc
 
 
 def vbatched_partition_lpt(h_n, ngpu: int):

@@ -60,6 +60,26 @@ static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d
   return (int)e;
 }
 
+
+// LAPACK DPOTRS on the vbatched factor: two side-'L' TRSMs (forward then backward substitution).
+static int potrs_impl(char uplo, const int* d_n, const int* d_nrhs, const double* const* dA,
+                      const int* d_ldda, double* const* dB, const int* d_lddb, int batch,
+                      int max_n, int max_nrhs, cudaStream_t stream) {
+  const bool up = (uplo == 'U' || uplo == 'u');
+  // 'L': L Y = B, L^T X = Y.  'U' (A = U^T U): U^T Y = B, U X = Y.
+  int rc = trsm_launch('L', up ? 'U' : 'L', up ? 'T' : 'N', 'N', d_n, d_nrhs, 1.0, dA, d_ldda, dB,
+                       d_lddb, batch, max_n, max_nrhs, stream);
+  if (rc != 0) return rc;
+  return trsm_launch('L', up ? 'U' : 'L', up ? 'N' : 'T', 'N', d_n, d_nrhs, 1.0, dA, d_ldda, dB,
+                     d_lddb, batch, max_n, max_nrhs, stream);
+}
+
+__global__ void nrhs_if_ok_kernel(const int* __restrict__ info, const int* __restrict__ nrhs,
+                                  int* __restrict__ out, int batch) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x)
+    out[i] = info[i] == 0 ? nrhs[i] : 0;
+}
+
 }  // namespace vb
 
 using namespace vb;
@@ -147,7 +167,7 @@ int vbatched_dtrsm(char side, char uplo, char transA, char diag, const int* d_m,
                    double alpha, const double* const* dA_array, const int* d_ldda,
                    double* const* dB_array, const int* d_lddb, int batchCount, int max_m,
                    int max_n, vb_stream_t stream) {
-  if (!(side == 'R' || side == 'r')) return -1;  // side 'L' is NEXT-2
+  if (!(side == 'R' || side == 'r' || side == 'L' || side == 'l')) return -1;
   if (!(uplo == 'L' || uplo == 'l' || uplo == 'U' || uplo == 'u')) return -2;
   if (!(transA == 'N' || transA == 'n' || transA == 'T' || transA == 't' || transA == 'C' || transA == 'c')) return -3;
   if (!(diag == 'N' || diag == 'n' || diag == 'U' || diag == 'u')) return -4;
@@ -157,6 +177,45 @@ int vbatched_dtrsm(char side, char uplo, char transA, char diag, const int* d_m,
   if (batchCount == 0) return 0;
   return trsm_launch(side, uplo, transA, diag, d_m, d_n, alpha, dA_array, d_ldda, dB_array, d_lddb,
                      batchCount, max_m, max_n, (cudaStream_t)stream);
+}
+
+int vbatched_dpotrs(char uplo, const int* d_n, const int* d_nrhs, const double* const* dA_array,
+                    const int* d_ldda, double* const* dB_array, const int* d_lddb, int batchCount,
+                    int max_n, int max_nrhs, vb_stream_t stream) {
+  if (!uplo_ok(uplo)) return -1;
+  if (batchCount < 0) return -8;
+  if (max_n < 0) return -9;
+  if (max_nrhs < 0) return -10;
+  if (batchCount == 0) return 0;
+  return potrs_impl(uplo, d_n, d_nrhs, dA_array, d_ldda, dB_array, d_lddb, batchCount, max_n,
+                    max_nrhs, (cudaStream_t)stream);
+}
+
+int vbatched_dposv(char uplo, const int* d_n, const int* d_nrhs, double* const* dA_array,
+                   const int* d_ldda, double* const* dB_array, const int* d_lddb, int* d_info,
+                   int batchCount, int max_n, int max_nrhs, vb_stream_t stream) {
+  if (!uplo_ok(uplo)) return -1;
+  if (batchCount < 0) return -9;
+  if (max_n < 0) return -10;
+  if (max_nrhs < 0) return -11;
+  if (batchCount == 0) return 0;
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, max_n, true, st);
+  if (rc != 0) return rc;
+  // matrices that failed (info != 0) keep B unchanged (LAPACK DPOSV): solve with nrhs = 0
+  void* ws = nullptr;
+  cudaError_t e = ws_alloc(&ws, sizeof(int) * (size_t)batchCount, st);
+  if (e != cudaSuccess) return (int)e;
+  int* nrhs_eff = static_cast<int*>(ws);
+  nrhs_if_ok_kernel<<<std::min((batchCount + 255) / 256, 1024), 256, 0, st>>>(d_info, d_nrhs,
+                                                                             nrhs_eff, batchCount);
+  e = cudaGetLastError();
+  if (e == cudaSuccess)
+    rc = potrs_impl(uplo, d_n, nrhs_eff, dA_array, d_ldda, dB_array, d_lddb, batchCount, max_n,
+                    max_nrhs, st);
+  cudaError_t e2 = ws_free(ws, st);
+  if (e != cudaSuccess) return (int)e;
+  return rc != 0 ? rc : (int)e2;
 }
 
 int vbatched_partition_lpt(const int* h_n, int batchCount, int ngpu, int* h_owner) {

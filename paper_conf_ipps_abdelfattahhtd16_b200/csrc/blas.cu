@@ -37,6 +37,7 @@ struct BlasArgs {
   int batch;
   // trsm
   bool tlower, unit, upper_in_A;
+  bool bt;  // trsm side 'L': the kernel solves the side-'R' problem on the transposed view of B
 };
 
 __device__ __forceinline__ int cdiv(int a, int b) { return (a + b - 1) / b; }
@@ -250,6 +251,12 @@ __device__ __forceinline__ double t_elem(const BlasArgs& a, const double* A, int
   return in_tri ? A[(size_t)aj * lda + ai] : 0.0;
 }
 
+// Element (r, c) of the right-hand side the kernel works on: B itself (side 'R') or B^T (side
+// 'L': op(A) X = alpha B  <=>  X^T op(A)^T = alpha B^T).
+__device__ __forceinline__ size_t bix(bool bt, int r, int c, int ldb) {
+  return bt ? (size_t)r * ldb + c : (size_t)c * ldb + r;
+}
+
 __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* off, int* counter) {
   __shared__ __align__(16) TrsmSmem s;
   __shared__ int s_t;
@@ -286,7 +293,7 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
         const int k0 = Kb * kTW, kw = min(kTW, n - k0);
         for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
           const int k = idx / kBT, i = idx % kBT;
-          s.x[k][i] = (k < kw && r0 + i < m) ? B[(size_t)(k0 + k) * ldb + r0 + i] : 0.0;
+          s.x[k][i] = (k < kw && r0 + i < m) ? B[bix(a.bt, r0 + i, k0 + k, ldb)] : 0.0;
         }
         for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
           const int j = idx / kTW, k = idx % kTW;
@@ -321,7 +328,7 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
       __syncthreads();
       for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
         const int k = idx / kBT, i = idx % kBT;
-        const double bv = (k < w && r0 + i < m) ? B[(size_t)(c0 + k) * ldb + r0 + i] : 0.0;
+        const double bv = (k < w && r0 + i < m) ? B[bix(a.bt, r0 + i, c0 + k, ldb)] : 0.0;
         s.x[k][i] = fma(a.alpha, bv, s.x[k][i]);
       }
       // inv(T_JJ): lane j of warp 0 computes column j by substitution
@@ -375,7 +382,7 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
             const int r = r0 + wr + x * 8 + g, c = wc + y * 8 + 2 * q + h;
-            if (r < m && c < w) B[(size_t)(c0 + c) * ldb + r] = xo[x][y][h];
+            if (r < m && c < w) B[bix(a.bt, r, c0 + c, ldb)] = xo[x][y][h];
           }
       __syncthreads();  // X_J visible to the CTA before the next block reads it
     }
@@ -447,16 +454,22 @@ int syrk_launch(char uplo, char trans, const int* d_n, const int* d_k, double al
   return launch_blas(a, stream);
 }
 
-int trsm_launch(char, char uplo, char ta, char diag, const int* d_m, const int* d_n, double alpha,
-                const double* const* dA, const int* d_lda, double* const* dB, const int* d_ldb,
-                int batch, int, int, cudaStream_t stream) {
+int trsm_launch(char side, char uplo, char ta, char diag, const int* d_m, const int* d_n,
+                double alpha, const double* const* dA, const int* d_lda, double* const* dB,
+                const int* d_ldb, int batch, int, int, cudaStream_t stream) {
   BlasArgs a = {};
   a.mode = kTrsm;
-  a.ta = is_t(ta);
+  // side 'L' = side 'R' on B^T with T = op(A)^T: flip the transposition, swap m and n
+  a.bt = (side == 'L' || side == 'l');
+  a.ta = is_t(ta) ^ a.bt;
   a.upper_in_A = (uplo == 'U' || uplo == 'u');
   a.tlower = (!a.upper_in_A) ^ a.ta;  // T = op(A) is lower iff (A lower) xor transposed
   a.unit = (diag == 'U' || diag == 'u');
-  a.m = d_m; a.n = d_n; a.k = d_n;
+  if (a.bt) {
+    a.m = d_n; a.n = d_m; a.k = d_m;
+  } else {
+    a.m = d_m; a.n = d_n; a.k = d_n;
+  }
   a.alpha = alpha; a.beta = 0.0;
   a.A = dA; a.lda = d_lda; a.C = dB; a.ldc = d_ldb;
   a.batch = batch;

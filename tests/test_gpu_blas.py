@@ -89,17 +89,19 @@ def test_syrk(uplo, trans):
             assert np.array_equal(got[other], C.get(i)[other])
 
 
+@pytest.mark.parametrize("side", ["R", "L"])
 @pytest.mark.parametrize("uplo", ["L", "U"])
 @pytest.mark.parametrize("ta", ["N", "T"])
 @pytest.mark.parametrize("diag", ["N", "U"])
-def test_trsm_right(uplo, ta, diag):
+def test_trsm(side, uplo, ta, diag):
     rng = np.random.default_rng(3)
     mn = [(0, 4), (1, 1), (5, 0), (70, 33), (64, 64), (130, 97), (3, 200), (257, 65)]
     m = [a for a, _ in mn]
     n = [b for _, b in mn]
-    A = Mats([(ni, ni) for ni in n], rng)
+    na = n if side == "R" else m  # order of the triangular A
+    A = Mats([(ni, ni) for ni in na], rng)
     # well-conditioned triangular: boost the diagonal
-    for i, ni in enumerate(n):
+    for i, ni in enumerate(na):
         if ni:
             blk = A.get(i)
             blk += 4 * np.eye(ni)
@@ -108,16 +110,16 @@ def test_trsm_right(uplo, ta, diag):
     A.dev.copy_(torch.from_numpy(A.host))
     B = Mats(list(zip(m, n)), rng)
     alpha = 0.75
-    vb.vbatched_dtrsm("R", uplo, ta, diag, _ints(m), _ints(n), alpha, A.ptrs, A.d_ld, B.ptrs, B.d_ld,
+    vb.vbatched_dtrsm(side, uplo, ta, diag, _ints(m), _ints(n), alpha, A.ptrs, A.d_ld, B.ptrs, B.d_ld,
                       len(m), max(m), max(n))
     torch.cuda.synchronize()
     out = B.result()
     for i in range(len(m)):
-        ref = oracle.dtrsm("R", uplo, ta, diag, alpha, A.get(i), B.get(i))
+        ref = oracle.dtrsm(side, uplo, ta, diag, alpha, A.get(i), B.get(i))
         got = B.get(i, out)
         if ref.size:
             scale = max(1.0, np.max(np.abs(ref)))
-            assert np.max(np.abs(got - ref)) / scale < 1e-12, (i, uplo, ta, diag)
+            assert np.max(np.abs(got - ref)) / scale < 1e-12, (i, side, uplo, ta, diag)
 
 
 def test_blas_argument_errors():
@@ -126,5 +128,5 @@ def test_blas_argument_errors():
     assert vb.vbatched_dgemm("N", "Q", z, z, z, 1, 0, z, 0, z, 0, 0, z, 1, 1, 1, 1, check=False) == -2
     assert vb.vbatched_dgemm("N", "N", z, z, z, 1, 0, z, 0, z, 0, 0, z, -1, 1, 1, 1, check=False) == -14
     assert vb.vbatched_dsyrk("Q", "N", z, z, 1, 0, z, 0, 0, z, 1, 1, 1, check=False) == -1
-    assert vb.vbatched_dtrsm("L", "L", "T", "N", z, z, 1, 0, z, 0, z, 1, 1, 1, check=False) == -1
+    assert vb.vbatched_dtrsm("X", "L", "T", "N", z, z, 1, 0, z, 0, z, 1, 1, 1, check=False) == -1
     assert vb.vbatched_dtrsm("R", "L", "T", "N", z, z, 1, 0, z, 0, z, 0, 1, 1, check=False) == 0

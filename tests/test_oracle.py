@@ -361,3 +361,47 @@ def test_trsm_oracle(side, uplo, ta, diag):
         ref = solve_triangular(opT.T, (2.0 * B).T, lower=np.allclose(opT.T, np.tril(opT.T))).T
         assert np.allclose(X @ opT, 2.0 * B, rtol=1e-12, atol=1e-12)
     assert np.allclose(X, ref, rtol=1e-12, atol=1e-12)
+
+
+# ---- NEXT-4: the solve (LAPACK DPOTRS / DPOSV) ------------------------------------------------
+@pytest.mark.parametrize("uplo", ["L", "U"])
+@pytest.mark.parametrize("n,nrhs", [(1, 1), (7, 3), (33, 5), (128, 1), (200, 17)])
+def test_potrs_oracle_exact_integer_family(uplo, n, nrhs):
+    """A = L L^T with integer unit-lower L (entries -1/0/1) and B = A X0 with integer X0:
+    every intermediate of both triangular solves is an integer below 2^53 and every division
+    is by 1, so the oracle must return X0 exactly (and the factor L exactly)."""
+    rng = np.random.default_rng(100 + n)
+    L = np.tril(rng.integers(-1, 2, size=(n, n)), -1).astype(np.int64) + np.eye(n, dtype=np.int64)
+    A = (L @ L.T).astype(np.float64)
+    X0 = rng.integers(-3, 4, size=(n, nrhs)).astype(np.int64)
+    B = (L @ (L.T @ X0)).astype(np.float64)
+    X, F, info = oracle.dposv(uplo, A, B)
+    assert info == 0
+    if uplo == "L":
+        assert np.array_equal(F, L.astype(np.float64))
+    else:
+        assert np.array_equal(F, L.T.astype(np.float64))
+    assert np.array_equal(X, X0.astype(np.float64))
+
+
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_potrs_oracle_residual_and_library(uplo):
+    """F1 matrices: the solution matches numpy's LAPACK solve (dgesv) to 1e-12 relative and the
+    residual ||A X - B|| is at rounding level."""
+    rng = np.random.default_rng(7)
+    for n, nrhs in [(5, 2), (64, 8), (257, 3)]:
+        A = vbgen.f1_matrix(9, n, n)
+        B = rng.standard_normal((n, nrhs))
+        X, _, info = oracle.dposv(uplo, A, B)
+        assert info == 0
+        ref = np.linalg.solve(A, B)
+        assert np.max(np.abs(X - ref)) <= 1e-12 * np.max(np.abs(ref))
+        assert np.linalg.norm(A @ X - B) <= 1e-13 * np.linalg.norm(A) * np.linalg.norm(X)
+
+
+def test_posv_oracle_failure_keeps_b():
+    A = vbgen.f1_matrix(9, 3, 40)
+    A[9, 9] = -A[9, 9]
+    B = np.arange(80, dtype=np.float64).reshape(40, 2)
+    X, _, info = oracle.dposv("L", A, B)
+    assert info == 10 and np.array_equal(X, B)
