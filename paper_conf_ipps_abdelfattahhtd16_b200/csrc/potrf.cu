@@ -1060,6 +1060,103 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
   }
 }
 
+// Look-ahead small-matrix kernel (32 < n <= ts, the default): the same 2-warp CTA and NB = 32
+// blocks as potrf_small_kernel, but the warps are specialised. Warp 0 owns the diagonal
+// blocks only (panel update of the diagonal block, POTF2, TRTRI); warp 1 owns every block
+// below the diagonal (panel update + TRSM + store). Warp 0 starts panel p+1 as soon as warp 1
+// has stored block 1 of panel p (the rows of the next diagonal block), so the pivot chain of
+// panel p+1 overlaps warp 1's remaining blocks of panel p. Named barriers (64 threads):
+//   1 inv_ready(p)  warp 0 arrives after TRTRI(p) (or on failure), warp 1 syncs before TRSM;
+//   2 block1(p)     warp 1 arrives after storing block 1 of panel p, warp 0 syncs before the
+//                   diagonal update of panel p+1;
+//   3 inv_free(p)   warp 1 arrives after its last TRSM of panel p, warp 0 syncs before it
+//                   overwrites s.inv with inv(L11) of panel p+1 (single inverse buffer).
+// Arrivals and syncs are paired under the same conditions (panel p has blocks below it and
+// did not fail), so no barrier phase is left open across matrices.
+template <bool UP>
+__global__ void __launch_bounds__(32 * kSmallWarps, 8)
+    potrf_small_la_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                          const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
+                          int range, int wait_upstream) {
+  __shared__ SmallSmem s;
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int g = lane >> 2, q = lane & 3;
+  for (;;) {
+    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
+    __syncthreads();
+    const int it = s.item;
+    __syncthreads();
+    if (it >= count) break;
+    const int m = order[start + it];
+    const int n = d_n[m], ld = d_ldda[m];
+    double* A = dA[m];
+    TL_BEGIN(t_tl)
+    const int npan = (n + 31) / 32;
+    if (warp == 0) {
+      bool pending_free = false;  // warp 1 will arrive inv_free for the previous panel
+      for (int p = 0; p < npan; ++p) {
+        const int j0 = 32 * p, nb = min(32, n - j0);
+        const bool below = p + 1 < npan;
+        if (p > 0) bar_group(2, 64);  // block 1 of panel p-1 (= these rows) is stored
+        double acc[4][4][2];
+        small_panel_update<UP>(acc, A, n, ld, j0, j0, nb, true, lane);
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < 4; ++nt) {
+            s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+            s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+          }
+        __syncwarp();
+        const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
+                                           s.wbuf, s.sv, s.tv);
+        if (pending_free) {  // warp 1 is done with inv(L11) of panel p-1
+          bar_group(3, 64);
+          pending_free = false;
+        }
+        if (info) {
+          if (lane == 0) {
+            s.info = info;
+            d_info[m] = j0 + info;
+          }
+          if (below) bar_group_arrive(1, 64);  // warp 1 reads s.info and stops
+          break;
+        }
+        if (!below) break;
+        trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
+        if (lane == 0) s.info = 0;
+        bar_group_arrive(1, 64);  // inv(L11) of panel p is ready
+        pending_free = true;
+      }
+    } else {
+      for (int p = 0; p + 1 < npan; ++p) {  // panels with blocks below the diagonal
+        const int j0 = 32 * p;
+        const int nblk = (n - j0 + 31) / 32;
+        double acc[4][4][2];
+        small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
+        bar_group(1, 64);  // inv(L11) of panel p (or the failure)
+        if (s.info) break;
+        small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane);
+        bar_group_arrive(2, 64);  // block 1 stored: warp 0 may start panel p+1
+        for (int b = 2; b < nblk; ++b) {
+          small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
+          small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
+        }
+        bar_group_arrive(3, 64);  // done with s.inv of panel p
+      }
+    }
+    __syncthreads();
+    if (tid == 0) s.info = 0;
+    TL_END(tid == 0, t_tl, m, 21)
+  }
+}
+
 // =======================================================================================
 // Warp-per-matrix kernel for 32 < n <= ts (replaces the 2-warp small kernel by default):
 // one warp factors one matrix alone — no inter-warp synchronisation — and 16 single-warp
@@ -1327,7 +1424,7 @@ static cudaError_t init_device_info() {
                                                     32 * (Cfg64d::WARPS + 1), sizeof(Smem2<Cfg64d>));
   if (e != cudaSuccess) return e;
   if (g_occ64 < 1) g_occ64 = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_kernel<false>,
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_la_kernel<false>,
                                                     32 * kSmallWarps, 0);
   if (e != cudaSuccess) return e;
   if (g_occ_small < 1) g_occ_small = 1;
@@ -1337,7 +1434,7 @@ static cudaError_t init_device_info() {
   if (g_occ_wsmall < 1) g_occ_wsmall = 1;
   {
     const char* v = getenv("VB_SMALL");
-    g_small = v ? atoi(v) : 2;
+    g_small = v ? atoi(v) : 3;
   }
   potrf_ts();
   g_num_sms = sms;
@@ -1371,7 +1468,13 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
     wait = 0;
   }
   if (max_n_hint > kWarpMaxN) {
-    if (g_small == 2) {
+    if (g_small == 3) {
+      cfg.blockDim = dim3(32 * kSmallWarps);
+      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
+      cfg.dynamicSmemBytes = 0;
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true> : potrf_small_la_kernel<false>,
+                             d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
+    } else if (g_small == 2) {
       cfg.blockDim = dim3(32 * kSmallWarps);
       cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
       cfg.dynamicSmemBytes = 0;
@@ -1401,7 +1504,7 @@ void potrf_occupancy(int* out4) {
   out4[0] = g_occ64;
   out4[1] = Cfg64d::WARPS;
   out4[2] = 0;  // (no separate NB=32 range)
-  out4[3] = g_small == 2 ? g_occ_small : g_occ_wsmall;
+  out4[3] = g_small >= 2 ? g_occ_small : g_occ_wsmall;
 }
 
 int potrf_num_launches(int max_n_hint) {
