@@ -454,10 +454,17 @@ def main():
         reference_arm(args, cfg, rank, world)
         return
     import torch
+    if os.environ.get("VB_BENCH_SHARE_GPU"):
+        # test hook: all ranks on cuda:0 with gloo collectives, to exercise the multi-rank
+        # path (shards, max-over-ranks time, info gather) on a one-GPU box. Never a bench value.
+        local_rank = 0
     if world > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if os.environ.get("VB_BENCH_SHARE_GPU"):
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
         our_arm(args, cfg, rank, world, local_rank)
     finally:
