@@ -15,7 +15,7 @@ class DeviceBatch:
     pointer array, n[], ldda[], info[] (int32), gidx[] (global matrix index for the hash)."""
 
     def __init__(self, n, ldda=None, seed=1, gidx=None, nonspd_mod=0, device="cuda",
-                 ldda_mode="pad32"):
+                 ldda_mode="pad32", dtype="f64"):
         self.n = np.ascontiguousarray(n, dtype=np.int32)
         self.B = len(self.n)
         self.ldda = np.ascontiguousarray(vbgen.ldda_for(self.n, ldda_mode) if ldda is None else ldda,
@@ -24,10 +24,13 @@ class DeviceBatch:
         self.seed = seed
         self.nonspd_mod = nonspd_mod
         self.device = torch.device(device)
-        self.off, total = vbgen.arena_layout(np.maximum(self.n, 0), self.ldda)
-        self.arena = torch.empty(total, dtype=torch.float64, device=self.device)
+        self.f32 = dtype == "f32"
+        es = 4 if self.f32 else 8
+        self.off, total = vbgen.arena_layout(np.maximum(self.n, 0), self.ldda, elem_bytes=es)
+        self.arena = torch.empty(total, dtype=torch.float32 if self.f32 else torch.float64,
+                                 device=self.device)
         base = self.arena.data_ptr()
-        self.ptrs_h = (base + 8 * self.off).astype(np.int64)
+        self.ptrs_h = (base + es * self.off).astype(np.int64)
         self.d_ptrs = torch.from_numpy(self.ptrs_h).to(self.device)
         self.d_n = torch.from_numpy(self.n).to(self.device)
         self.d_ldda = torch.from_numpy(self.ldda).to(self.device)
@@ -36,7 +39,7 @@ class DeviceBatch:
 
     def fill(self, poison=False, stream=None, uplo="L"):
         s = torch.cuda.current_stream().cuda_stream if stream is None else stream
-        flags = (1 if poison else 0) | (2 if uplo == "U" else 0)
+        flags = (1 if poison else 0) | (2 if uplo == "U" else 0) | (4 if self.f32 else 0)
         vbdev.fill_f1(self.seed, self.B, self.d_n.data_ptr(), self.d_ldda.data_ptr(),
                       self.d_ptrs.data_ptr(), self.d_gidx.data_ptr(), self.nonspd_mod, flags, s)
         return self
@@ -45,9 +48,15 @@ class DeviceBatch:
         """Write a host matrix into slot i: its lower ('L') or upper ('U') triangle; the other
         strict triangle and the padding rows get the NaN poison."""
         n, ld = int(self.n[i]), int(self.ldda[i])
-        blk = np.full((ld, n), np.nan)
-        if poison:
-            blk.view(np.uint64)[:] = np.uint64(vbgen.NAN_POISON_BITS)
+        if self.f32:
+            blk = np.full((ld, n), np.nan, dtype=np.float32)
+            if poison:
+                blk.view(np.uint32)[:] = np.uint32(0x7FC0BEEF)
+            A = np.asarray(A, dtype=np.float32)
+        else:
+            blk = np.full((ld, n), np.nan)
+            if poison:
+                blk.view(np.uint64)[:] = np.uint64(vbgen.NAN_POISON_BITS)
         tri = np.tril(np.ones((n, n), bool)) if uplo == "L" else np.triu(np.ones((n, n), bool))
         blk[:n, :n] = np.where(tri, A, blk[:n, :n])
         t = torch.from_numpy(blk.ravel(order="F").copy())
@@ -67,10 +76,12 @@ class DeviceBatch:
         return self.d_info[: self.B].cpu().numpy()
 
     def dpotrf(self, max_n=None, stream=None, uplo="L", check=True):
-        from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf
+        """vbatched_dpotrf (or vbatched_spotrf for an FP32 batch) on the whole batch."""
+        from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf, vbatched_spotrf
         mx = int(self.n.max()) if (max_n is None and self.B) else (max_n or 0)
-        return vbatched_dpotrf(uplo, self.d_n, self.d_ptrs, self.d_ldda, self.d_info, self.B, mx,
-                               stream=stream, check=check)
+        fn = vbatched_spotrf if self.f32 else vbatched_dpotrf
+        return fn(uplo, self.d_n, self.d_ptrs, self.d_ldda, self.d_info, self.B, mx,
+                  stream=stream, check=check)
 
     def host_matrix_input(self, i) -> np.ndarray:
         """The matrix the generator writes for slot i (numpy twin)."""

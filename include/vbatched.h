@@ -66,6 +66,17 @@ typedef struct CUstream_st* vb_stream_t; /* == cudaStream_t */
 int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
                     int* d_info, int batchCount, int max_n, vb_stream_t stream);
 
+/* vbatched_spotrf — the same factorisation of FP32 matrices (the paper
+ * tests single precision too). Arguments, layout, uplo, info codes and
+ * ownership exactly as vbatched_dpotrf with float storage. B200 has no exact-FP32 tensor-core
+ * MMA, so the kernels load FP32, compute in FP64 on the DMMA tensor cores (pivots, updates and
+ * TRSM in FP64) and store the factor rounded to FP32; each stored column is re-read in FP32 by
+ * later panels. Results are therefore at least as accurate as an FP32 LAPACK SPOTRF; info
+ * follows the FP64 pivot test (!(p > 0)). ldda_i that is not a multiple of 4 (16 bytes) takes the
+ * cp.async staging path instead of TMA bulk copies. */
+int vbatched_spotrf(char uplo, const int* d_n, float* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream);
+
 /* LAPACK-like interface: identical to vbatched_dpotrf but max_n is not
  * needed; the device scan computes it (no host synchronisation: launch sizes assume the
  * worst case and idle CTAs exit). Argument numbers as above; there is no check -7. */

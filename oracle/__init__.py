@@ -43,6 +43,8 @@ def lib():
         build()
         L = ctypes.CDLL(LIB_PATH)
         L.oracle_dpotrf_lower.argtypes = [ctypes.c_int, _dp, ctypes.c_int]
+        L.oracle_spotrf_lower.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_float), ctypes.c_int]
+        L.oracle_spotrf_lower.restype = ctypes.c_int
         L.oracle_dpotrf_lower.restype = ctypes.c_int
         L.oracle_dpotrf_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip, _ip, ctypes.c_int]
         L.oracle_dpotrf_batch.restype = None
@@ -83,6 +85,21 @@ def dpotrf(a: np.ndarray) -> tuple[np.ndarray, int]:
     assert out.shape == (n, n)
     info = lib().oracle_dpotrf_lower(n, _ptr(out), max(1, n))
     return out, info
+
+
+def spotrf(a: np.ndarray) -> tuple[np.ndarray, int]:
+    """Oracle Cholesky of one FP32 matrix (float arithmetic, same recurrence as dpotrf)."""
+    out = np.array(a, dtype=np.float32, order="F", copy=True)
+    n = out.shape[0]
+    assert out.shape == (n, n)
+    info = lib().oracle_spotrf_lower(n, out.ctypes.data_as(ctypes.POINTER(ctypes.c_float)), max(1, n))
+    return out, info
+
+
+def backward_error_f32(A0: np.ndarray, L: np.ndarray, info: int) -> float:
+    """||A - L L^T||_F / (nb ||A||_F eps32), eps32 = 2^-24, long double (the FP32 reading of
+    SURVEY.md §8(c) #13)."""
+    return backward_error(np.asarray(A0, np.float64), np.asarray(L, np.float64), info) * 2.0 ** -29
 
 
 def dpotrf_inplace(buf: np.ndarray, n: int, ld: int) -> int:

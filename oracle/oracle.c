@@ -18,6 +18,9 @@
  *    info = j+1 (1-based) at the first pivot that is not > 0 (NaN counts as failure); the
  *    failing pivot value is stored at (j,j) and the routine stops. Pinned by
  *    tests/test_oracle.py (closed forms, exact integer families, MKL, exact rationals).
+ *  - oracle_spotrf_lower: the same recurrence in IEEE single precision (float arithmetic,
+ *    sqrtf correctly rounded, no contraction) — the FP32 problem of SURVEY.md §8(f) NEXT-3
+ *    (the paper's SP runs; LAPACK SPOTRF).
  *  - oracle_dpotrf_batch: the vbatched problem (§III-A: each matrix has
  *    its own size and leading dimension) = the single-matrix oracle applied to each matrix;
  *    OpenMP dynamic over matrices (one core per matrix, the paper's CPU scheme,
@@ -69,6 +72,41 @@ int oracle_dpotrf_lower(int n, double* a, int lda) {
   }
   /* Copy back: computed columns (all rows), plus the failing pivot. Columns after a
    * failure are left as they were in a (LAPACK stops there). */
+  for (int j = 0; j < done; ++j)
+    for (int i = j; i < n; ++i) a[IDX(i, j, lda)] = w[(size_t)i * n + j];
+  if (info > 0) a[IDX(info - 1, info - 1, lda)] = w[(size_t)(info - 1) * n + (info - 1)];
+  free(w);
+  return info;
+}
+
+/* oracle_dpotrf_lower in IEEE single precision (same order of operations). */
+int oracle_spotrf_lower(int n, float* a, int lda) {
+  if (n <= 0) return 0;
+  float* w = (float*)malloc(sizeof(float) * (size_t)n * (size_t)n);
+  if (!w) return -1000;
+  for (int i = 0; i < n; ++i)
+    for (int j = 0; j <= i; ++j) w[(size_t)i * n + j] = a[IDX(i, j, lda)];
+  int info = 0;
+  int done = n;
+  for (int j = 0; j < n; ++j) {
+    const float* lj = w + (size_t)j * n;
+    float s = w[(size_t)j * n + j];
+    for (int k = 0; k < j; ++k) s = s - lj[k] * lj[k];
+    if (!(s > 0.0f)) {
+      w[(size_t)j * n + j] = s;
+      info = j + 1;
+      done = j;
+      break;
+    }
+    const float ljj = sqrtf(s);
+    w[(size_t)j * n + j] = ljj;
+    for (int i = j + 1; i < n; ++i) {
+      const float* li = w + (size_t)i * n;
+      float t = li[j];
+      for (int k = 0; k < j; ++k) t = t - li[k] * lj[k];
+      w[(size_t)i * n + j] = t / ljj;
+    }
+  }
   for (int j = 0; j < done; ++j)
     for (int i = j; i < n; ++i) a[IDX(i, j, lda)] = w[(size_t)i * n + j];
   if (info > 0) a[IDX(info - 1, info - 1, lda)] = w[(size_t)(info - 1) * n + (info - 1)];

@@ -34,7 +34,8 @@ cudaError_t ws_free(void* p, cudaStream_t stream) { return cudaFreeAsync(p, stre
 
 static bool uplo_ok(char u) { return u == 'L' || u == 'l' || u == 'U' || u == 'u'; }
 
-static int potrf_impl(char uplo, const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+template <typename E>
+static int potrf_impl(char uplo, const int* d_n, E* const* dA, const int* d_ldda, int* d_info,
                       int batch, int max_n, bool check_max, cudaStream_t stream) {
   if (!uplo_ok(uplo)) return -1;
   const bool up = (uplo == 'U' || uplo == 'u');
@@ -87,6 +88,12 @@ using namespace vb;
 extern "C" {
 
 int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream) {
+  return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, max_n, true,
+                    (cudaStream_t)stream);
+}
+
+int vbatched_spotrf(char uplo, const int* d_n, float* const* dA_array, const int* d_ldda,
                     int* d_info, int batchCount, int max_n, vb_stream_t stream) {
   return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, max_n, true,
                     (cudaStream_t)stream);

@@ -65,6 +65,19 @@ VB_DEVINL void cp_async8(void* sdst, const void* gsrc, bool pred) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),
                "r"(pred ? 8 : 0));
 }
+// cp.async 4 bytes with zero fill when !pred.
+VB_DEVINL void cp_async4(void* sdst, const void* gsrc, bool pred) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),
+               "r"(pred ? 4 : 0));
+}
+// cp.async of one element of the storage type (double or float).
+template <typename E>
+VB_DEVINL void cp_async_e(E* sdst, const E* gsrc, bool pred) {
+  if constexpr (sizeof(E) == 8)
+    cp_async8(sdst, gsrc, pred);
+  else
+    cp_async4(sdst, gsrc, pred);
+}
 // cp.async 16 bytes (L2 only), zero fill when !pred.
 VB_DEVINL void cp_async16(void* sdst, const void* gsrc, bool pred) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(sdst)), "l"(gsrc),

@@ -18,10 +18,16 @@ cudaError_t launch_scan_bin(const int* d_n, const int* d_ldda, int* d_info, int 
 cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
                                bool up, cudaStream_t stream);
+// FP32 storage (SPOTRF): the same kernels with float loads/stores, FP64 arithmetic inside.
+cudaError_t launch_potrf_paths(const int* d_n, float* const* dA, const int* d_ldda, int* d_info,
+                               int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
+                               bool up, cudaStream_t stream);
 
 int potrf_num_launches(int max_n_hint);
 // max_n <= 32: one warp kernel that validates and factors directly (no scan).
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                                int batch, int max_n, bool up, cudaStream_t stream);
+cudaError_t launch_potrf_direct(const int* d_n, float* const* dA, const int* d_ldda, int* d_info,
                                 int batch, int max_n, bool up, cudaStream_t stream);
 void potrf_occupancy(int* out4);  // blocked CTAs/SM, blocked compute warps, 0, small CTAs/SM
 

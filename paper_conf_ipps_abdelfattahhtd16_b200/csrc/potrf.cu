@@ -289,8 +289,8 @@ VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, dou
 // pivot). Blocked 16 + 16: POTF2 of columns 0..15 with all 32 rows in registers (which also
 // produces L21), the trailing 16x16 update C22 -= L21 L21^T on DMMA, POTF2 of C22.
 // sv/tv (>= 32 doubles) receive l_cc and 1/l_cc. Returns info.
-template <bool UP>
-VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, int lda,
+template <bool UP, typename E = double>
+VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, E* Ag, int lda,
                             double* ws, double* sv, double* tv) {
   const int nb1 = min(nb, 16), nb2 = nb - nb1;
   int info;
@@ -352,7 +352,7 @@ VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, double* Ag, in
     for (int c = 0; c < 16; ++c) a[c] = (c < nb2 && r < nb2) ? T22[c * ldt + r] : selp(c == r, 1.0, 0.0);
     const int info2 = potf2_regs_warp<16>(a, nb2, lane, ws, sv + 16, tv + 16);
     const int ncol = info2 ? info2 : nb2;
-    double* A22 = Ag + (size_t)16 * lda + 16;
+    E* A22 = Ag + (size_t)16 * lda + 16;
 #pragma unroll
     for (int c = 0; c < 16; ++c)
       if (lane < 16 && c < ncol && r >= c && r < nb2) {
@@ -396,19 +396,26 @@ VB_DEVINL void bar_group_arrive(int id, int nthreads) {
 // Blocked kernel (n > ts) building blocks: warp w owns 16 full rows of each MB-row block, so
 // the TRSM runs from registers and stores straight to global; the TMA stage ring is not
 // aliased with anything, so the producer keeps prefetching across row blocks and panels.
-template <int NB_, int KC_, int STAGES_, int MINB_, int WARPS_ = 8>
+// E: the matrices' storage type (double for DPOTRF, float for SPOTRF); the ring stages hold E,
+// everything from the fragments on is FP64 (DMMA). Ring leading dims padded so that the
+// fragment loads are bank-conflict free (+4 doubles / +8 floats).
+template <int NB_, int KC_, int STAGES_, int MINB_, int WARPS_ = 8, typename E_ = double>
 struct Cfg2 {
+  using E = E_;
   static constexpr int NB = NB_, KC = KC_, STAGES = STAGES_, MINB = MINB_;
   static constexpr int WARPS = WARPS_;       // compute warps (16 rows each)
   static constexpr int THREADS = 32 * WARPS, MB = 16 * WARPS, NT = NB / 8;
-  static constexpr int LDA = MB + 4, LDB = NB + 4, LDT = NB + 4;
+  static constexpr int PAD = sizeof(E_) == 8 ? 4 : 8;
+  static constexpr int LDA = MB + PAD, LDB = NB + PAD, LDT = NB + 4;
+  static constexpr int G = 16 / (int)sizeof(E_);  // elements per 16 bytes (bulk-copy granule)
 };
 using Cfg64d = Cfg2<64, 16, 2, 3, 4>;  // v3, 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer
+using Cfg64s = Cfg2<64, 16, 2, 3, 4, float>;  // the same for FP32 storage (SPOTRF)
 
 template <class C>
 struct Smem2 {
-  double a[C::STAGES][C::KC][C::LDA];  // A chunk: [k][row]
-  double b[C::STAGES][C::KC][C::LDB];  // B chunk: [k][panel row]
+  alignas(16) typename C::E a[C::STAGES][C::KC][C::LDA];  // A chunk: [k][row]
+  alignas(16) typename C::E b[C::STAGES][C::KC][C::LDB];  // B chunk: [k][panel row]
   // Diagonal block T[c][r]. After diag_block64v2: T11 slot = inv(L22) as B operand,
   // T12 slot (cols 32..63, rows 0..31) = inv(L11) as B operand, T21 = L21, T22 = L22.
   double T[C::NB][C::LDT];
@@ -428,7 +435,8 @@ struct Smem2 {
 // L21 = C21 inv(L11)^T -> T21, C22 -= L21 L21^T, L22 = potf2(C22), inv(L22) -> T11.
 // Stores L11, L21, L22 (rows < nb) to global (Ad, ld). Sets s.info (1-based, in-block).
 template <class CC, bool UP>
-__device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int lane, double* Ad,
+__device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int lane,
+                                            typename CC::E* Ad,
                                             int ld, bool below) {
   constexpr int LDT = CC::LDT;
   double* T = &s.T[0][0];
@@ -503,23 +511,28 @@ __device__ __noinline__ void diag_block64v2(Smem2<CC>& s, int nb, int wg, int la
 
 // Producer (warp 0): chunk kc of the row block at r0 into ring slot gi % STAGES.
 template <class C, bool UP>
-VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, int n, int ld,
-                            int r0, int j0, int lane, bool bulk) {
+VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::E* A, int n,
+                            int ld, int r0, int j0, int lane, bool bulk) {
+  using E = typename C::E;
+  constexpr int G = C::G;
   const int st = gi % C::STAGES;
   const uint32_t u = gi / C::STAGES;
   const int k0 = kc * C::KC;
   if (lane == 0 && u > 0) mbar_wait(&s.empty[st], (u - 1) & 1);
   __syncwarp();
   if (bulk) {
-    const int ra = (min(C::MB, n - r0) + 1) & ~1;
-    const int rb = (min(C::NB, n - j0) + 1) & ~1;
-    if (lane == 0) mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * 8));
+    // segments rounded up to 16 bytes: the extra rows lie inside ldda (ldda is a multiple of
+    // G here) and only ever feed output rows/columns that are never stored
+    const int ra = (min(C::MB, n - r0) + G - 1) / G * G;
+    const int rb = (min(C::NB, n - j0) + G - 1) / G * G;
+    if (lane == 0)
+      mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * (int)sizeof(E)));
     __syncwarp();
     if (lane < C::KC) {
-      bulk_g2s(&s.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * 8, &s.full[st]);
+      bulk_g2s(&s.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * sizeof(E), &s.full[st]);
     } else if (lane >= 16 && lane < 16 + C::KC) {
       const int c = lane - 16;
-      bulk_g2s(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * 8, &s.full[st]);
+      bulk_g2s(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * sizeof(E), &s.full[st]);
     }
   } else {
     // Odd ldda / unaligned base ('L'), or uplo 'U': the chunk is gathered with 8-byte cp.async
@@ -533,26 +546,26 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const double* A, i
 #pragma unroll 4
       for (int r = lane >> 4; r < C::MB; r += 2) {
         const bool p = r0 + r < n;
-        cp_async8(&s.a[st][c][r], A + (p ? (size_t)(r0 + r) * ld + k0 + c : 0), p);
+        cp_async_e<E>(&s.a[st][c][r], A + (p ? (size_t)(r0 + r) * ld + k0 + c : 0), p);
       }
 #pragma unroll 4
       for (int r = lane >> 4; r < C::NB; r += 2) {
         const bool p = j0 + r < n;
-        cp_async8(&s.b[st][c][r], A + (p ? (size_t)(j0 + r) * ld + k0 + c : 0), p);
+        cp_async_e<E>(&s.b[st][c][r], A + (p ? (size_t)(j0 + r) * ld + k0 + c : 0), p);
       }
     } else {
 #pragma unroll 4
       for (int c = 0; c < C::KC; ++c) {
-        const double* col = A + (size_t)(k0 + c) * ld;
+        const E* col = A + (size_t)(k0 + c) * ld;
 #pragma unroll
         for (int r = lane; r < C::MB; r += 32) {
           const bool p = r0 + r < n;
-          cp_async8(&s.a[st][c][r], p ? col + r0 + r : A, p);
+          cp_async_e<E>(&s.a[st][c][r], p ? col + r0 + r : A, p);
         }
 #pragma unroll
         for (int r = lane; r < C::NB; r += 32) {
           const bool p = j0 + r < n;
-          cp_async8(&s.b[st][c][r], p ? col + j0 + r : A, p);
+          cp_async_e<E>(&s.b[st][c][r], p ? col + j0 + r : A, p);
         }
       }
     }
@@ -645,10 +658,12 @@ VB_DEVINL void trsm_regs64(Smem2<CC>& s, double (&acc)[2][8][2], int lane) {
 // panel's L), so TMA never reads a column before it is final.
 
 template <class C, bool UP>
-VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int lane,
+VB_DEVINL void produce_matrix3(Smem2<C>& s, const typename C::E* A, int n, int ld, int lane,
                                uint32_t& gchunk, uint32_t& gpanel) {
   constexpr int NB = C::NB, MB = C::MB, KC = C::KC;
-  const bool bulk = !UP && ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((ld & 1) == 0);
+  using E = typename C::E;
+  constexpr int G = C::G;
+  const bool bulk = !UP && ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && (ld % G == 0);
   const int npan = (n + NB - 1) / NB;
   int done = npan;  // panels the consumers will complete for this matrix
   fence_proxy_async();
@@ -659,8 +674,8 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
     // at the panel boundary. Everything after them reads panel p-1's columns.
     const int nk_free = (j0 - NB) / KC;
     if (bulk && lane < min(NB, n - j0)) {
-      const int rn = (min(MB, n - j0) + 1) & ~1;
-      bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + j0, rn * 8);
+      const int rn = (min(MB, n - j0) + G - 1) / G * G;
+      bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + j0, rn * (int)sizeof(E));
     }
     for (int kc = 0; kc < nk_free; ++kc) issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
     if (lane == 0) mbar_wait(&s.panel_done, (gpanel + p - 1) & 1);  // panel p-1 is stored
@@ -671,8 +686,8 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const double* A, int n, int ld, int 
     }
     for (int r0 = j0; r0 < n; r0 += MB) {
       if (r0 > j0 && bulk && lane < min(NB, n - j0)) {  // warm L2 with this block's panel values
-        const int rn = (min(MB, n - r0) + 1) & ~1;
-        bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * 8);
+        const int rn = (min(MB, n - r0) + G - 1) / G * G;
+        bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * (int)sizeof(E));
       }
       for (int kc = (r0 == j0 ? nk_free : 0); kc < nk; ++kc)
         issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
@@ -696,9 +711,9 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
       for (int kk = 0; kk < C::KC / 4; ++kk) {
         double fa[2], fb[NTL];
 #pragma unroll
-        for (int mt = 0; mt < 2; ++mt) fa[mt] = -s.a[st][kk * 4 + q][wrow + mt * 8 + g];
+        for (int mt = 0; mt < 2; ++mt) fa[mt] = -(double)s.a[st][kk * 4 + q][wrow + mt * 8 + g];
 #pragma unroll
-        for (int nt = 0; nt < NTL; ++nt) fb[nt] = s.b[st][kk * 4 + q][nt * 8 + g];
+        for (int nt = 0; nt < NTL; ++nt) fb[nt] = (double)s.b[st][kk * 4 + q][nt * 8 + g];
 #pragma unroll
         for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
@@ -716,7 +731,7 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
 }
 
 template <class C, bool UP>
-VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int ld,
+VB_DEVINL void consume_matrix3(Smem2<C>& s, typename C::E* __restrict__ A, int n, int ld,
                                int* info_out, uint32_t& gchunk, uint32_t& gpanel) {
   constexpr int NB = C::NB, MB = C::MB, KC = C::KC, STAGES = C::STAGES, NT = C::NT;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -845,7 +860,7 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, double* __restrict__ A, int n, int l
 
 template <class C, bool UP>
 __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
-    potrf_blocked3_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+    potrf_blocked3_kernel(const int* __restrict__ d_n, typename C::E* const* __restrict__ dA,
                           const int* __restrict__ d_ldda, int* __restrict__ d_info,
                           const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
                           int range, int wait_upstream) {
@@ -909,8 +924,8 @@ struct SmallSmem {
 };
 
 // acc (32 x 32 block at rows r0.., cols j0..) = A - L[r0:, 0:j0] L[j0:j0+32, 0:j0]^T
-template <bool UP>
-VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restrict__ A, int n,
+template <bool UP, typename E = double>
+VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ A, int n,
                                   int ld, int r0, int j0, int nb, bool diag, int lane) {
   const int g = lane >> 2, q = lane & 3;
 #pragma unroll
@@ -946,8 +961,8 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const double* __restri
 
 // X = C inv(L11)^T for a 32 x 32 block in registers (inv[k][n] upper in k,n: zero blocks
 // skipped), then direct stores of rows < n.
-template <bool UP>
-VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], double* __restrict__ A,
+template <bool UP, typename E = double>
+VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], E* __restrict__ A,
                                 int n, int ld, int r0, int j0, int lane) {
   const int g = lane >> 2, q = lane & 3;
   double x[4][4][2];
@@ -1073,9 +1088,9 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
 //                   overwrites s.inv with inv(L11) of panel p+1 (single inverse buffer).
 // Arrivals and syncs are paired under the same conditions (panel p has blocks below it and
 // did not fail), so no barrier phase is left open across matrices.
-template <bool UP>
+template <bool UP, typename E = double>
 __global__ void __launch_bounds__(32 * kSmallWarps, 8)
-    potrf_small_la_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+    potrf_small_la_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                           const int* __restrict__ d_ldda, int* __restrict__ d_info,
                           const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
                           int range, int wait_upstream) {
@@ -1095,7 +1110,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     if (it >= count) break;
     const int m = order[start + it];
     const int n = d_n[m], ld = d_ldda[m];
-    double* A = dA[m];
+    E* A = dA[m];
     TL_BEGIN(t_tl)
     const int npan = (n + 31) / 32;
     if (warp == 0) {
@@ -1309,8 +1324,8 @@ struct WarpSmem {
 };
 
 // One matrix (n <= NM) by one warp, rows in registers: one HBM read, one HBM write.
-template <int NM, bool UP>
-VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* info_out, int lane,
+template <int NM, bool UP, typename E = double>
+VB_DEVINL void potrf_warp_matrix(E* __restrict__ A, int n, int ld, int* info_out, int lane,
                                  double* ws, double* sv, double* tv) {
   double a[NM];
 #pragma unroll
@@ -1329,9 +1344,9 @@ VB_DEVINL void potrf_warp_matrix(double* __restrict__ A, int n, int ld, int* inf
 // wait_upstream: 1 when launched directly after the scan (the only factorisation kernel),
 // 0 when launched after a blocked kernel (whose CTAs passed the scan's completion before
 // releasing this grid, so the scan's outputs are already visible).
-template <bool UP>
+template <bool UP, typename E = double>
 __global__ void __launch_bounds__(32 * kWarpsPerCta)
-    potrf_warp_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+    potrf_warp_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                       const int* __restrict__ d_ldda, int* __restrict__ d_info,
                       const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
                       int wait_upstream) {
@@ -1350,11 +1365,11 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
     const int n = d_n[m], ld = d_ldda[m];
     TL_BEGIN(t_tl)
     if (n <= 8)
-      potrf_warp_matrix<8, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<8, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else if (n <= 16)
-      potrf_warp_matrix<16, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<16, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else
-      potrf_warp_matrix<32, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<32, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     TL_END(lane == 0, t_tl, m, 40)
   }
 }
@@ -1362,9 +1377,9 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 // Direct warp path for batches whose max_n <= 32 (no scan, no sort: with every matrix this
 // small there is nothing to balance): warp w validates (info -2/-4/-7, as the scan would) and
 // factors matrices w, w + nwarps, ... One launch per call — the latency path for C1.
-template <bool UP>
+template <bool UP, typename E = double>
 __global__ void __launch_bounds__(32 * kWarpsPerCta)
-    potrf_warp_direct_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
+    potrf_warp_direct_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                              const int* __restrict__ d_ldda, int* __restrict__ d_info, int batch,
                              int max_n) {
   __shared__ WarpSmem s;
@@ -1379,11 +1394,11 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
     if (lane == 0) d_info[m] = code;
     if (code != 0 || n == 0) continue;
     if (n <= 8)
-      potrf_warp_matrix<8, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<8, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else if (n <= 16)
-      potrf_warp_matrix<16, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<16, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     else
-      potrf_warp_matrix<32, UP>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
+      potrf_warp_matrix<32, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
   }
 }
 
@@ -1406,6 +1421,23 @@ int potrf_ts() {
   return g_ts;
 }
 
+template <class C>
+static cudaError_t setup_blocked(int* occ) {
+  cudaError_t e = cudaFuncSetAttribute(potrf_blocked3_kernel<C, false>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)sizeof(Smem2<C>));
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(potrf_blocked3_kernel<C, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<C>));
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked3_kernel<C, false>,
+                                                    32 * (C::WARPS + 1), sizeof(Smem2<C>));
+  if (*occ < 1) *occ = 1;
+  return e;
+}
+
+static int g_occ64s = 0;
+
 static cudaError_t init_device_info() {
   if (g_num_sms) return cudaSuccess;
   int dev;
@@ -1414,16 +1446,8 @@ static cudaError_t init_device_info() {
   int sms = 0;
   e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d, false>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64d>));
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(potrf_blocked3_kernel<Cfg64d, true>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<Cfg64d>));
-  if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ64, potrf_blocked3_kernel<Cfg64d, false>,
-                                                    32 * (Cfg64d::WARPS + 1), sizeof(Smem2<Cfg64d>));
-  if (e != cudaSuccess) return e;
-  if (g_occ64 < 1) g_occ64 = 1;
+  if ((e = setup_blocked<Cfg64d>(&g_occ64)) != cudaSuccess) return e;
+  if ((e = setup_blocked<Cfg64s>(&g_occ64s)) != cudaSuccess) return e;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_la_kernel<false>,
                                                     32 * kSmallWarps, 0);
   if (e != cudaSuccess) return e;
@@ -1441,12 +1465,26 @@ static cudaError_t init_device_info() {
   return cudaSuccess;
 }
 
+template <typename E>
+struct BlockedCfgOf;
+template <>
+struct BlockedCfgOf<double> {
+  using C = Cfg64d;
+};
+template <>
+struct BlockedCfgOf<float> {
+  using C = Cfg64s;
+};
+
 // One persistent grid per non-empty size range, chained with programmatic dependent launch
 // (each grid releases the next as soon as it starts, so the next range's CTAs take the SMs
-// the previous kernel frees at its tail).
-cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
-                               int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
-                               bool up, cudaStream_t stream) {
+// the previous kernel frees at its tail). E = storage type (double: DPOTRF, float: SPOTRF; the
+// arithmetic is FP64 in both).
+template <typename E>
+static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda, int* d_info,
+                                int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
+                                bool up, cudaStream_t stream) {
+  using C = typename BlockedCfgOf<E>::C;
   cudaError_t e = init_device_info();
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -1458,34 +1496,35 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.stream = stream;
   int wait = 1;  // the first factorisation kernel after the scan waits for it
   if (max_n_hint > g_ts) {
-    cfg.blockDim = dim3(32 * (Cfg64d::WARPS + 1));
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ64)));
-    cfg.dynamicSmemBytes = sizeof(Smem2<Cfg64d>);
-    e = cudaLaunchKernelEx(&cfg, up ? potrf_blocked3_kernel<Cfg64d, true>
-                                    : potrf_blocked3_kernel<Cfg64d, false>,
+    const int occ = sizeof(E) == 8 ? g_occ64 : g_occ64s;
+    cfg.blockDim = dim3(32 * (C::WARPS + 1));
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * occ)));
+    cfg.dynamicSmemBytes = sizeof(Smem2<C>);
+    e = cudaLaunchKernelEx(&cfg, up ? potrf_blocked3_kernel<C, true> : potrf_blocked3_kernel<C, false>,
                            d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
   if (max_n_hint > kWarpMaxN) {
-    if (g_small == 3) {
-      cfg.blockDim = dim3(32 * kSmallWarps);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
-      cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true> : potrf_small_la_kernel<false>,
-                             d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-    } else if (g_small == 2) {
-      cfg.blockDim = dim3(32 * kSmallWarps);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
-      cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true> : potrf_small_kernel<false>, d_n,
-                             dA, d_ldda, d_info, ctrl, order, 1, wait);
+    cfg.blockDim = dim3(32 * kSmallWarps);
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
+    cfg.dynamicSmemBytes = 0;
+    if constexpr (sizeof(E) == 8) {
+      if (g_small == 3) {
+        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true> : potrf_small_la_kernel<false>,
+                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
+      } else if (g_small == 2) {
+        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true> : potrf_small_kernel<false>, d_n,
+                               dA, d_ldda, d_info, ctrl, order, 1, wait);
+      } else {
+        cfg.blockDim = dim3(32);
+        cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
+        e = cudaLaunchKernelEx(&cfg, up ? potrf_wsmall_kernel<true> : potrf_wsmall_kernel<false>,
+                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
+      }
     } else {
-      cfg.blockDim = dim3(32);
-      cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
-      cfg.dynamicSmemBytes = 0;
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_wsmall_kernel<true> : potrf_wsmall_kernel<false>, d_n,
-                             dA, d_ldda, d_info, ctrl, order, 1, wait);
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true, E> : potrf_small_la_kernel<false, E>,
+                             d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
     }
     if (e != cudaSuccess) return e;
     wait = 0;
@@ -1495,8 +1534,19 @@ cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_l
   cfg.gridDim = dim3(std::max(1, std::min((warps + kWarpsPerCta - 1) / kWarpsPerCta,
                                           g_num_sms * 8)));
   cfg.dynamicSmemBytes = 0;
-  return cudaLaunchKernelEx(&cfg, up ? potrf_warp_kernel<true> : potrf_warp_kernel<false>, d_n, dA,
-                            d_ldda, d_info, ctrl, order, wait);
+  return cudaLaunchKernelEx(&cfg, up ? potrf_warp_kernel<true, E> : potrf_warp_kernel<false, E>,
+                            d_n, dA, d_ldda, d_info, ctrl, order, wait);
+}
+
+cudaError_t launch_potrf_paths(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                               int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
+                               bool up, cudaStream_t stream) {
+  return launch_paths<double>(d_n, dA, d_ldda, d_info, batch, max_n_hint, ctrl, order, up, stream);
+}
+cudaError_t launch_potrf_paths(const int* d_n, float* const* dA, const int* d_ldda, int* d_info,
+                               int batch, int max_n_hint, const Ctrl* ctrl, const int* order,
+                               bool up, cudaStream_t stream) {
+  return launch_paths<float>(d_n, dA, d_ldda, d_info, batch, max_n_hint, ctrl, order, up, stream);
 }
 
 void potrf_occupancy(int* out4) {
@@ -1513,18 +1563,27 @@ int potrf_num_launches(int max_n_hint) {
   return 3 + (max_n_hint > potrf_ts() ? 1 : 0);
 }
 
-cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
-                                int batch, int max_n, bool up, cudaStream_t stream) {
+template <typename E>
+static cudaError_t launch_direct(const int* d_n, E* const* dA, const int* d_ldda, int* d_info,
+                                 int batch, int max_n, bool up, cudaStream_t stream) {
   cudaError_t e = init_device_info();
   if (e != cudaSuccess) return e;
   const int grid = std::max(1, std::min((batch + kWarpsPerCta - 1) / kWarpsPerCta, g_num_sms * 16));
   if (up)
-    potrf_warp_direct_kernel<true><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info,
-                                                                          batch, max_n);
+    potrf_warp_direct_kernel<true, E><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda,
+                                                                             d_info, batch, max_n);
   else
-    potrf_warp_direct_kernel<false><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda, d_info,
-                                                                           batch, max_n);
+    potrf_warp_direct_kernel<false, E><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda,
+                                                                              d_info, batch, max_n);
   return cudaGetLastError();
+}
+cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
+                                int batch, int max_n, bool up, cudaStream_t stream) {
+  return launch_direct<double>(d_n, dA, d_ldda, d_info, batch, max_n, up, stream);
+}
+cudaError_t launch_potrf_direct(const int* d_n, float* const* dA, const int* d_ldda, int* d_info,
+                                int batch, int max_n, bool up, cudaStream_t stream) {
+  return launch_direct<float>(d_n, dA, d_ldda, d_info, batch, max_n, up, stream);
 }
 
 }  // namespace vb

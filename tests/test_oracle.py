@@ -405,3 +405,40 @@ def test_posv_oracle_failure_keeps_b():
     B = np.arange(80, dtype=np.float64).reshape(40, 2)
     X, _, info = oracle.dposv("L", A, B)
     assert info == 10 and np.array_equal(X, B)
+
+
+# ---- NEXT-3: the FP32 oracle (oracle_spotrf_lower) --------------------------------------------
+def test_spotrf_oracle_exact_families():
+    """min(i,j) -> tril(ones) and integer unit-lower L (entries -1/0/1, A = L L^T below 2^24):
+    every operation is exact in FP32 too, so the factor must be bit-exact."""
+    n = 120
+    i = np.arange(1, n + 1)
+    L, info = oracle.spotrf(np.minimum.outer(i, i).astype(np.float32))
+    assert info == 0 and np.array_equal(np.tril(L), np.tril(np.ones((n, n), np.float32)))
+    rng = np.random.default_rng(41)
+    for n in (17, 64, 100):
+        Li = np.tril(rng.integers(-1, 2, size=(n, n)), -1).astype(np.int64) + np.eye(n, dtype=np.int64)
+        A = (Li @ Li.T)
+        assert np.abs(A).max() < 2 ** 24
+        L, info = oracle.spotrf(A.astype(np.float32))
+        assert info == 0 and np.array_equal(np.tril(L), Li.astype(np.float32))
+
+
+def test_spotrf_oracle_vs_fp64_and_lapack():
+    """On F1 matrices (kappa ~ 1.6) the FP32 factor is within a small multiple of n eps32 of the
+    FP64 oracle's (row-scaled) and of numpy's float32 LAPACK Cholesky; the FP32 backward error
+    ratio stays <= 10; an injected negative pivot gives the same info as FP64."""
+    for n in (5, 64, 300):
+        A = vbgen.f1_matrix(13, n, n)
+        A32 = A.astype(np.float32)
+        L32, info = oracle.spotrf(A32)
+        L64, info64 = oracle.dpotrf(A32.astype(np.float64))
+        assert info == info64 == 0
+        rs = oracle.rowscaled_diff(L32.astype(np.float64), L64, n)
+        assert rs <= 4 * n * 2.0 ** -24, (n, rs)
+        Ln = np.linalg.cholesky(A32)
+        assert oracle.rowscaled_diff(L32.astype(np.float64), Ln.astype(np.float64), n) <= 4 * n * 2.0 ** -24
+        assert oracle.backward_error_f32(A32, np.tril(L32), info) <= 10.0
+    A = vbgen.f1_matrix(13, 7, 90).astype(np.float32)
+    A[40, 40] = -A[40, 40]
+    assert oracle.spotrf(A)[1] == 41

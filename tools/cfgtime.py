@@ -13,6 +13,7 @@ from harness import DeviceBatch  # noqa: E402
 reps = int(os.environ.get("REPS", "5"))
 tag = os.environ.get("TAG", "")
 uplo = os.environ.get("UPLO", "L")
+dtype = os.environ.get("DTYPE", "f64")
 for cfg in sys.argv[1:]:
     if cfg.startswith("u"):
         nn, cnt = (int(x) for x in cfg[1:].split("x"))
@@ -20,7 +21,7 @@ for cfg in sys.argv[1:]:
     else:
         c = vbgen.CONFIGS[cfg]
         n, seed, mod = vbgen.sizes(cfg), c.seed, c.nonspd_mod
-    db = DeviceBatch(n, seed=seed, nonspd_mod=mod)
+    db = DeviceBatch(n, seed=seed, nonspd_mod=mod, dtype=dtype)
     ts = []
     for it in range(reps + 1):
         db.fill(uplo=uplo)

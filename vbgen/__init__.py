@@ -141,11 +141,11 @@ def ldda_for(n: np.ndarray, mode: str = "pad32") -> np.ndarray:
     raise ValueError(mode)
 
 
-def arena_layout(n: np.ndarray, ldda: np.ndarray, align_bytes: int = 256):
+def arena_layout(n: np.ndarray, ldda: np.ndarray, align_bytes: int = 256, elem_bytes: int = 8):
     """Element offsets of each matrix in one arena (each base `align_bytes`-aligned) and the
     total element count."""
     sz = ldda.astype(np.int64) * np.maximum(n.astype(np.int64), 0)
-    al = align_bytes // 8
+    al = align_bytes // elem_bytes
     sz_al = (sz + al - 1) // al * al
     off = np.zeros(len(n), dtype=np.int64)
     if len(n) > 1:

@@ -10,7 +10,9 @@
 //     Writes the lower triangle (and, if poison bit 0 is set, NaN-payload sentinels into the
 //     strict upper triangle and the padding rows n..ldda-1). Poison bit 1 selects upper
 //     storage instead (the same symmetric matrix in the upper triangle, for uplo 'U'; the
-//     sentinels then go to the strict lower triangle). Returns a cudaError_t.
+//     sentinels then go to the strict lower triangle). Poison bit 2: the matrices are FP32
+//     (d_A holds float*; each value is the F1 double rounded to nearest float, the poison
+//     becomes a float NaN with a payload). Returns a cudaError_t.
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -39,10 +41,11 @@ __global__ void fill_f1_kernel(uint64_t seed, int batch, const int* __restrict__
     int kneg = -1;
     if (nonspd_mod > 0 && (int)(g % (uint64_t)nonspd_mod) == nonspd_mod - 1)
       kneg = (int)(splitmix64(s0 ^ g ^ 0x5EEDull) % (uint64_t)n);
-    const bool up = (poison & 2) != 0, poi = (poison & 1) != 0;
+    const bool up = (poison & 2) != 0, poi = (poison & 1) != 0, f32 = (poison & 4) != 0;
     const int rows = poi ? ld : n;
     for (int j = 0; j < n; ++j) {
       double* col = A + (size_t)j * ld;
+      float* colf = reinterpret_cast<float*>(A) + (size_t)j * ld;
       const int i0 = (poi || up) ? 0 : j, i1 = (up && !poi) ? j + 1 : rows;
       for (int i = i0 + threadIdx.x; i < i1; i += blockDim.x) {
         double v;
@@ -57,7 +60,10 @@ __global__ void fill_f1_kernel(uint64_t seed, int batch, const int* __restrict__
         } else {
           v = __longlong_as_double((long long)kPoison);
         }
-        col[i] = v;
+        if (f32)
+          colf[i] = v == v ? (float)v : __int_as_float(0x7FC0BEEF);
+        else
+          col[i] = v;
       }
     }
   }
