@@ -54,6 +54,9 @@ def parse():
                    help="profiling only: keep the first B matrices of the config")
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--precision", default="d", choices=["d", "s"],
+                   help="d: vbatched_dpotrf (the headline); s: vbatched_spotrf (FP32 storage, "
+                        "FP64 arithmetic; no e2e / CPU legs)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=8.0,
                    help="target wall seconds of the bounded oracle sample")
@@ -251,7 +254,12 @@ def our_arm(args, cfg, rank, world, local_rank):
     from paper_conf_ipps_abdelfattahhtd16_b200 import shard
     mine = shard.shard_indices(n_all, world, rank)  # LPT on n^3/3, identical on every rank
     n_loc = n_all[mine]
-    db = DeviceBatch(n_loc, seed=cfg.seed, gidx=mine, nonspd_mod=cfg.nonspd_mod, device=dev)
+    single = args.precision == "s"
+    if single:
+        args.no_e2e = True
+        args.no_cpu_baseline = True
+    db = DeviceBatch(n_loc, seed=cfg.seed, gidx=mine, nonspd_mod=cfg.nonspd_mod, device=dev,
+                     dtype="f32" if single else "f64")
     ws = torch.empty(vb.vbatched_dpotrf_workspace_size(db.B), dtype=torch.uint8, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
@@ -265,16 +273,21 @@ def our_arm(args, cfg, rank, world, local_rank):
     def step(ev):
         # the product call: scan and factorisation kernels chained with PDL on one stream
         ev[0].record(stream)
-        vb.vbatched_dpotrf("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, db.B, max_n, stream=stream)
+        db.dpotrf(max_n=max_n, stream=stream)  # vbatched_dpotrf (or vbatched_spotrf)
         ev[1].record(stream)
 
     def step_split(ev):
         # the same kernels through the two-phase API, an event between the scan and the
         # factorisation launches: the factorisation kernels' own duration (roofline)
         ev[0].record(stream)
-        vb.vbatched_dpotrf_scan("L", db.d_n, db.d_ldda, db.d_info, db.B, max_n, ws, stream)
-        ev[1].record(stream)
-        vb.vbatched_dpotrf_factor("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, db.B, max_n, ws, stream)
+        if single:  # no two-phase API for FP32: the whole call (scan included) is timed
+            ev[1].record(stream)
+            db.dpotrf(max_n=max_n, stream=stream)
+        else:
+            vb.vbatched_dpotrf_scan("L", db.d_n, db.d_ldda, db.d_info, db.B, max_n, ws, stream)
+            ev[1].record(stream)
+            vb.vbatched_dpotrf_factor("L", db.d_n, db.d_ptrs, db.d_ldda, db.d_info, db.B, max_n,
+                                      ws, stream)
         ev[2].record(stream)
 
     def barrier():
@@ -308,7 +321,7 @@ def our_arm(args, cfg, rank, world, local_rank):
     scan_ms = [e[0].elapsed_time(e[1]) for e in evk]
     info = db.info()
     ok_local = vbgen.expected_flops(n_loc[info == 0])
-    alg_bytes_local = vbgen.algorithmic_bytes(n_loc[info == 0])
+    alg_bytes_local = vbgen.algorithmic_bytes(n_loc[info == 0]) * (0.5 if single else 1.0)
     # global info[] from every rank's (index, info) pairs; flops count only info == 0 matrices
     info_all = shard.gather_info(len(n_all), mine, info, device=dev)
     bad_info = int(np.sum(info_all != expected_info(cfg, n_all, np.arange(len(n_all)))))
@@ -334,7 +347,7 @@ def our_arm(args, cfg, rank, world, local_rank):
         achieved = alg_bytes_local / kern_avg_s / 1e9
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "peak_source": src}
-    tr = load_traffic(cfg.name)
+    tr = load_traffic(cfg.name + ("_s" if single else ""))
     roof["traffic"] = tr.get("bytes_per_launch") if tr else None
     if tr:
         roof["traffic_source"] = tr.get("source")
@@ -363,9 +376,11 @@ def our_arm(args, cfg, rank, world, local_rank):
 
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world,
+            "metric": METRIC if not single else METRIC.replace("DPOTRF", "SPOTRF"),
+            "value": value, "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": max_total_ms / args.steps,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64" if not single else "f64 (f32 storage)",
             "data": "synthetic", "config": config_dict(cfg, world),
             "roofline": roof, "cpu_baseline": cpu, "cpu_lapack": cpu_lapack, "e2e": e2e,
             "gpu_launches": launches_per_step * args.steps, "clocks": clocks,
