@@ -923,10 +923,10 @@ struct SmallSmem {
   int info;
 };
 
-// acc (32 x 32 block at rows r0.., cols j0..) = A - L[r0:, 0:j0] L[j0:j0+32, 0:j0]^T
+// acc (32 x 32 block at rows r0.., cols j0..) = A (its lower part when diag)
 template <bool UP, typename E = double>
-VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ A, int n,
-                                  int ld, int r0, int j0, int nb, bool diag, int lane) {
+VB_DEVINL void small_acc_init(double (&acc)[4][4][2], const E* __restrict__ A, int n, int ld,
+                              int r0, int j0, int nb, bool diag, int lane) {
   const int g = lane >> 2, q = lane & 3;
 #pragma unroll
   for (int mt = 0; mt < 4; ++mt)
@@ -938,6 +938,13 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ 
         const bool v = row < n && col < j0 + nb && (!diag || row >= col);
         acc[mt][nt][h] = v ? __ldcg(A + gix<UP>(row, col, ld)) : 0.0;
       }
+}
+
+// acc -= L[r0:r0+32, kb:ke] L[j0:j0+32, kb:ke]^T, fragments straight from L2 (k ascending)
+template <bool UP, typename E = double>
+VB_DEVINL void small_kloop(double (&acc)[4][4][2], const E* __restrict__ A, int n, int ld,
+                           int r0, int j0, int kb, int ke, int lane) {
+  const int g = lane >> 2, q = lane & 3;
   bool rv[4], cv[4];
 #pragma unroll
   for (int t = 0; t < 4; ++t) {
@@ -945,7 +952,7 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ 
     cv[t] = j0 + t * 8 + g < n;
   }
 #pragma unroll 2
-  for (int k = q; k < j0; k += 4) {
+  for (int k = kb + q; k < ke; k += 4) {
     double fa[4], fb[4];
 #pragma unroll
     for (int t = 0; t < 4; ++t) {
@@ -957,6 +964,14 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ 
 #pragma unroll
       for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
   }
+}
+
+// acc (32 x 32 block at rows r0.., cols j0..) = A - L[r0:, 0:j0] L[j0:j0+32, 0:j0]^T
+template <bool UP, typename E = double>
+VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ A, int n,
+                                  int ld, int r0, int j0, int nb, bool diag, int lane) {
+  small_acc_init<UP, E>(acc, A, n, ld, r0, j0, nb, diag, lane);
+  small_kloop<UP, E>(acc, A, n, ld, r0, j0, 0, j0, lane);
 }
 
 // X = C inv(L11)^T for a 32 x 32 block in registers (inv[k][n] upper in k,n: zero blocks
@@ -1118,9 +1133,15 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
       for (int p = 0; p < npan; ++p) {
         const int j0 = 32 * p, nb = min(32, n - j0);
         const bool below = p + 1 < npan;
-        if (p > 0) bar_group(2, 64);  // block 1 of panel p-1 (= these rows) is stored
         double acc[4][4][2];
-        small_panel_update<UP>(acc, A, n, ld, j0, j0, nb, true, lane);
+        small_acc_init<UP, E>(acc, A, n, ld, j0, j0, nb, true, lane);
+        if (p > 0) {
+          // columns of the panels before p-1 are final: their update runs while warp 1 is
+          // still on block 1 of panel p-1; the newest 32 columns after block 1 is stored
+          small_kloop<UP, E>(acc, A, n, ld, j0, j0, 0, j0 - 32, lane);
+          bar_group(2, 64);  // block 1 of panel p-1 (= these rows) is stored
+          small_kloop<UP, E>(acc, A, n, ld, j0, j0, j0 - 32, j0, lane);
+        }
 #pragma unroll
         for (int mt = 0; mt < 4; ++mt)
 #pragma unroll
