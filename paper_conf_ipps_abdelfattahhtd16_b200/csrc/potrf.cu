@@ -529,10 +529,14 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
       mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * (int)sizeof(E)));
     __syncwarp();
     if (lane < C::KC) {
-      bulk_g2s(&s.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * sizeof(E), &s.full[st]);
+      // A rows stream (re-read only a panel later): evict first; the panel rows are re-read
+      // for every row block of the panel: evict last (C5 DRAM traffic and time)
+      bulk_g2s_hint(&s.a[st][lane][0], A + (size_t)(k0 + lane) * ld + r0, ra * sizeof(E),
+                    &s.full[st], policy_evict_first());
     } else if (lane >= 16 && lane < 16 + C::KC) {
       const int c = lane - 16;
-      bulk_g2s(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * sizeof(E), &s.full[st]);
+      bulk_g2s_hint(&s.b[st][c][0], A + (size_t)(k0 + c) * ld + j0, rb * sizeof(E), &s.full[st],
+                    policy_evict_last());
     }
   } else {
     // Odd ldda / unaligned base ('L'), or uplo 'U': the chunk is gathered with 8-byte cp.async
