@@ -54,6 +54,9 @@ def parse():
                    help="profiling only: keep the first B matrices of the config")
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--graph", action="store_true",
+                   help="time replays of a CUDA graph that captured one vbatched_dpotrf call "
+                        "(SURVEY.md §8(d): the launch-latency-free variant for C1/C2)")
     p.add_argument("--precision", default="d", choices=["d", "s"],
                    help="d: vbatched_dpotrf (the headline); s: vbatched_spotrf (FP32 storage, "
                         "FP64 arithmetic; no e2e / CPU legs)")
@@ -298,6 +301,21 @@ def our_arm(args, cfg, rank, world, local_rank):
         prepare()
         step([torch.cuda.Event(enable_timing=True) for _ in range(2)])
     torch.cuda.synchronize()
+    if args.graph:
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            db.dpotrf(max_n=max_n)  # captured on the graph's stream (workspace alloc/free nodes too)
+        torch.cuda.synchronize()
+
+        def step(ev):  # noqa: F811 — the timed step becomes one graph replay
+            ev[0].record(stream)
+            graph.replay()
+            ev[1].record(stream)
+
+        for _ in range(args.warmup):
+            prepare()
+            step([torch.cuda.Event(enable_timing=True) for _ in range(2)])
+        torch.cuda.synchronize()
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
     sampler = ClockSampler(local_rank)
     barrier()
@@ -390,6 +408,8 @@ def our_arm(args, cfg, rank, world, local_rank):
         }
         if args.batch_limit:
             line["config"]["batch_limit"] = args.batch_limit
+        if args.graph:
+            line["config"]["launch"] = "CUDA graph replay of one vbatched_dpotrf call"
         print(json.dumps(line), flush=True)
 
 

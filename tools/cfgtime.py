@@ -15,7 +15,12 @@ tag = os.environ.get("TAG", "")
 uplo = os.environ.get("UPLO", "L")
 dtype = os.environ.get("DTYPE", "f64")
 for cfg in sys.argv[1:]:
-    if cfg.startswith("u"):
+    if "x" in cfg and cfg.startswith("C"):  # e.g. C2x4: config C2's distribution, 4x the batch
+        base, mult = cfg.split("x")
+        c0 = vbgen.CONFIGS[base]
+        c = vbgen.Config(cfg, c0.batch * int(mult), c0.dist, c0.nmax, c0.seed, c0.nonspd_mod)
+        n, seed, mod = vbgen.sizes(c), c.seed, c.nonspd_mod
+    elif cfg.startswith("u"):
         nn, cnt = (int(x) for x in cfg[1:].split("x"))
         n, seed, mod = np.full(cnt, nn, dtype=np.int32), 3, 0
     else:
