@@ -108,9 +108,10 @@ __device__ __forceinline__ int find_matrix(const int* off, int batch, int t) {
 
 // ---------------------------------------------------------------------------------------
 // GEMM / SYRK tile: C[r0:r0+64, c0:c0+64] = alpha op(A) op(B) + beta C (masked for SYRK).
+constexpr int kGStages = 3;  // cp.async ring depth: one CTA barrier per k chunk
 struct GemmSmem {
-  double a[2][kBK][kLD];  // [k][row]
-  double b[2][kBK][kLD];  // [k][col]
+  double a[kGStages][kBK][kLD];  // [k][row]
+  double b[kGStages][kBK][kLD];  // [k][col]
 };
 
 __device__ __forceinline__ void gemm_stage(GemmSmem& s, int st, const double* A, int lda, bool ta,
@@ -139,9 +140,10 @@ __device__ __forceinline__ void gemm_stage(GemmSmem& s, int st, const double* A,
   }
 }
 
-__global__ void __launch_bounds__(kGThreads) gemm_syrk_kernel(BlasArgs a, const int* off,
-                                                              int* counter) {
-  __shared__ __align__(16) GemmSmem s;
+__global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, const int* off,
+                                                                 int* counter) {
+  extern __shared__ __align__(16) unsigned char gsm_raw[];
+  GemmSmem& s = *reinterpret_cast<GemmSmem*>(gsm_raw);
   __shared__ int s_t;
   pdl_wait();
   const int total = off[a.batch];
@@ -190,13 +192,16 @@ __global__ void __launch_bounds__(kGThreads) gemm_syrk_kernel(BlasArgs a, const 
     const int nk = cdiv(K, kBK);
     if (nk > 0) gemm_stage(s, 0, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, 0);
     cp_async_commit();
+    if (nk > 1) gemm_stage(s, 1, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, kBK);
+    cp_async_commit();
     for (int kc = 0; kc < nk; ++kc) {
-      if (kc + 1 < nk)
-        gemm_stage(s, (kc + 1) & 1, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, (kc + 1) * kBK);
+      cp_async_wait<1>();  // chunk kc has landed (only chunk kc+1 may still be in flight)
+      __syncthreads();     // ... for every thread; and every warp is done with chunk kc-1
+      if (kc + 2 < nk)
+        gemm_stage(s, (kc + 2) % kGStages, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0,
+                   (kc + 2) * kBK);
       cp_async_commit();
-      cp_async_wait<1>();
-      __syncthreads();
-      const int st = kc & 1;
+      const int st = kc % kGStages;
 #pragma unroll
       for (int kk = 0; kk < kBK / 4; ++kk) {
         double fa[4], fb[4];
@@ -209,9 +214,9 @@ __global__ void __launch_bounds__(kGThreads) gemm_syrk_kernel(BlasArgs a, const 
 #pragma unroll
           for (int y = 0; y < 4; ++y) dmma(acc[x][y], fa[x], fb[y]);
       }
-      __syncthreads();
     }
     cp_async_wait<0>();
+    __syncthreads();  // the next tile's prologue refills stages 0 and 1
     double* C = a.C[mi];
     const int ldc = a.ldc[mi];
 #pragma unroll
@@ -396,6 +401,8 @@ int launch_blas(const BlasArgs& a, cudaStream_t stream) {
     int dev;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(gemm_syrk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(GemmSmem));
   }
   void* ws = nullptr;
   cudaError_t e = ws_alloc(&ws, sizeof(int) * ((size_t)a.batch + 2), stream);
@@ -414,8 +421,13 @@ int launch_blas(const BlasArgs& a, cudaStream_t stream) {
     cfg.stream = stream;
     cfg.blockDim = dim3(kGThreads);
     cfg.gridDim = dim3(g_sms * 8);
-    if (a.mode == kTrsm) e = cudaLaunchKernelEx(&cfg, trsm_kernel, a, (const int*)off, counter);
-    else e = cudaLaunchKernelEx(&cfg, gemm_syrk_kernel, a, (const int*)off, counter);
+    if (a.mode == kTrsm) {
+      e = cudaLaunchKernelEx(&cfg, trsm_kernel, a, (const int*)off, counter);
+    } else {
+      cfg.gridDim = dim3(g_sms * 4);  // 4 CTAs per SM (registers, 52 KB smem each)
+      cfg.dynamicSmemBytes = sizeof(GemmSmem);
+      e = cudaLaunchKernelEx(&cfg, gemm_syrk_kernel, a, (const int*)off, counter);
+    }
   }
   cudaError_t e2 = ws_free(ws, stream);
   return (int)(e != cudaSuccess ? e : e2);
