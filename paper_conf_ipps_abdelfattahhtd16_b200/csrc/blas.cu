@@ -243,9 +243,11 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
 constexpr int kTW = 32;
 struct TrsmSmem {
   double x[kTW][kLD];     // A operand [k][row]
-  double t[kTW][kTW + 4];  // B operand [k][col]
-  double d[kTW][kTW + 1];  // raw diagonal block T_JJ [row][col]
+  double t[kTW][kTW + 4];  // B operand [k][col]; scratch for the transposed inverse
+  double d[kTW][kTW + 1];  // diagonal block T_JJ as the lower factor L of TRTRI: d[c][r] = L[r][c]
   double inv[kTW][kTW + 4];  // inv(T_JJ) [k][col]
+  double S[16 * LDS_T];      // TRTRI scratch
+  double tv[kTW];            // 1 / L[c][c]
 };
 
 __device__ __forceinline__ double t_elem(const BlasArgs& a, const double* A, int lda, int i, int j) {
@@ -326,9 +328,13 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
         for (int y = 0; y < 2; ++y)
 #pragma unroll
           for (int h = 0; h < 2; ++h) s.x[wc + y * 8 + 2 * q + h][wr + x * 8 + g] = -acc[x][y][h];
+      // TRTRI input L (lower, L[r][c] at d[c][r]): L = T_JJ when T is lower, L = T_JJ^T when
+      // it is upper (then inv(L)^T = inv(T_JJ) comes out of TRTRI directly)
       for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
         const int j = idx / kTW, i = idx % kTW;
-        s.d[i][j] = (i < w && j < w) ? t_elem(a, A, lda, c0 + i, c0 + j) : (i == j ? 1.0 : 0.0);
+        const double v = (i < w && j < w) ? t_elem(a, A, lda, c0 + i, c0 + j) : (i == j ? 1.0 : 0.0);
+        if (a.tlower) s.d[j][i] = v;
+        else s.d[i][j] = v;
       }
       __syncthreads();
       for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
@@ -336,31 +342,18 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
         const double bv = (k < w && r0 + i < m) ? B[bix(a.bt, r0 + i, c0 + k, ldb)] : 0.0;
         s.x[k][i] = fma(a.alpha, bv, s.x[k][i]);
       }
-      // inv(T_JJ): lane j of warp 0 computes column j by substitution
+      // inv(T_JJ) by warp 0: 8x8 substitution + recursive doubling on DMMA (trtri32_dmma_warp)
+      // into the B-operand layout INV[k][n] = inv(L)[n][k]; for a lower T that is inv(T)^T,
+      // transposed once through s.t
       if (warp == 0) {
-        const int j = lane;
-        double xcol[kTW];
-        if (!a.tlower) {  // upper: x_i = 0 (i>j), x_j = 1/d_jj, x_i = -(sum_{k=i+1..j} d_ik x_k)/d_ii
-#pragma unroll
-          for (int i = kTW - 1; i >= 0; --i) {
-            double acc2 = 0.0;
-#pragma unroll
-            for (int k = i + 1; k < kTW; ++k) acc2 = fma(s.d[i][k], xcol[k], acc2);
-            const double r = 1.0 / s.d[i][i];
-            xcol[i] = (i > j) ? 0.0 : (i == j ? r : -acc2 * r);
-          }
-        } else {
-#pragma unroll
-          for (int i = 0; i < kTW; ++i) {
-            double acc2 = 0.0;
-#pragma unroll
-            for (int k = 0; k < i; ++k) acc2 = fma(s.d[i][k], xcol[k], acc2);
-            const double r = 1.0 / s.d[i][i];
-            xcol[i] = (i < j) ? 0.0 : (i == j ? r : -acc2 * r);
-          }
+        s.tv[lane] = 1.0 / s.d[lane][lane];
+        __syncwarp();
+        double* out = a.tlower ? &s.t[0][0] : &s.inv[0][0];
+        trtri32_dmma_warp(&s.d[0][0], kTW + 1, s.tv, out, kTW + 4, s.S, LDS_T, lane);
+        if (a.tlower) {
+#pragma unroll 4
+          for (int k = 0; k < kTW; ++k) s.inv[k][lane] = s.t[lane][k];
         }
-#pragma unroll
-        for (int i = 0; i < kTW; ++i) s.inv[i][j] = xcol[i];
       }
       __syncthreads();
       double xo[4][2][2];

@@ -91,7 +91,6 @@ VB_DEVINL unsigned long long tl_now() {
 #define TL_END(pred, v, m, kind)
 #endif
 
-constexpr int LDS_T = 18;  // TRTRI32 scratch leading dim (16 columns used)
 
 // ---------------------------------------------------------------------------------------
 // POTF2 of an nb x nb (nb <= NM <= 32) lower block by one warp, lane r holding row r in
@@ -165,125 +164,6 @@ VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws_, do
 }
 
 // ---------------------------------------------------------------------------------------
-// Inverse of a 32x32 lower-triangular L (T[c*ldt+r] = L[r][c], tv[c] = 1/L[c][c]) by one
-// warp: 8x8 diagonal blocks by substitution (lane = block column), then two levels of
-// recursive doubling inv([[A,0],[B,C]]) = [[inv A, 0], [-inv C B inv A, inv C]] on DMMA.
-// Output INV[k*ldi + n] = X[n][k], X = L^-1 (the TRSM's B operand layout); the 32x32 block
-// of INV is fully written (zeros above the diagonal of X). S: 16 x LDS_T x 2 doubles with
-// leading dimension lds.
-VB_DEVINL void trtri32_dmma_warp(const double* T, int ldt, const double* tv, double* INV,
-                                 int ldi, double* S, int lds, int lane) {
-  const int g = lane >> 2, q = lane & 3;
-  for (int e = lane; e < 32 * 32; e += 32) INV[(e >> 5) * ldi + (e & 31)] = 0.0;
-  __syncwarp();
-  {  // level 0: column c of inv(D_b), D_b = L[8b:8b+8, 8b:8b+8]
-    const int b = lane >> 3, c = lane & 7, o = 8 * b;
-    double x[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      double s = 0.0;
-#pragma unroll
-      for (int k = 0; k < i; ++k) s = fma(T[(o + k) * ldt + o + i], x[k], s);
-      const double r = tv[o + i];
-      x[i] = (i < c) ? 0.0 : ((i == c) ? r : -s * r);
-    }
-#pragma unroll
-    for (int i = 0; i < 8; ++i) INV[(o + c) * ldi + o + i] = x[i];
-  }
-  __syncwarp();
-  // level 1: blocks (2p, 2p+1), p = 0, 1: X[16p+8:, 16p:16p+8] = -inv(D_{2p+1}) B inv(D_{2p})
-  {
-    double t[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
-#pragma unroll
-    for (int p = 0; p < 2; ++p) {
-      const int o = 16 * p;
-#pragma unroll
-      for (int ks = 0; ks < 2; ++ks) {
-        const double a = T[(o + ks * 4 + q) * ldt + o + 8 + g];  // B[g][k]
-        const double bb = INV[(o + g) * ldi + o + ks * 4 + q];   // invA[k][g]
-        dmma(t[p], a, bb);
-      }
-    }
-#pragma unroll
-    for (int p = 0; p < 2; ++p) {
-      S[(p * 8 + g) * lds + 2 * q] = t[p][0];
-      S[(p * 8 + g) * lds + 2 * q + 1] = t[p][1];
-    }
-    __syncwarp();
-    double r[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
-#pragma unroll
-    for (int p = 0; p < 2; ++p) {
-      const int o = 16 * p;
-#pragma unroll
-      for (int ks = 0; ks < 2; ++ks) {
-        const double a = INV[(o + 8 + ks * 4 + q) * ldi + o + 8 + g];  // invC[g][k]
-        const double bb = S[(p * 8 + ks * 4 + q) * lds + g];            // Tm[k][g]
-        dmma(r[p], a, bb);
-      }
-    }
-#pragma unroll
-    for (int p = 0; p < 2; ++p) {
-      const int o = 16 * p;
-      INV[(o + 2 * q) * ldi + o + 8 + g] = -r[p][0];
-      INV[(o + 2 * q + 1) * ldi + o + 8 + g] = -r[p][1];
-    }
-  }
-  __syncwarp();
-  // level 2: X[16:32, 0:16] = -inv(C16) L[16:32, 0:16] inv(A16)
-  {
-    double t[2][2][2];
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt) t[mt][nt][0] = t[mt][nt][1] = 0.0;
-#pragma unroll
-    for (int ks = 0; ks < 4; ++ks) {
-      double a[2], bb[2];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt) a[mt] = T[(ks * 4 + q) * ldt + 16 + mt * 8 + g];
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt) bb[nt] = INV[(nt * 8 + g) * ldi + ks * 4 + q];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 2; ++nt) dmma(t[mt][nt], a[mt], bb[nt]);
-    }
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt) {
-        S[(mt * 8 + g) * lds + nt * 8 + 2 * q] = t[mt][nt][0];
-        S[(mt * 8 + g) * lds + nt * 8 + 2 * q + 1] = t[mt][nt][1];
-      }
-    __syncwarp();
-    double r[2][2][2];
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt) r[mt][nt][0] = r[mt][nt][1] = 0.0;
-#pragma unroll
-    for (int ks = 0; ks < 4; ++ks) {
-      double a[2], bb[2];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt) a[mt] = INV[(16 + ks * 4 + q) * ldi + 16 + mt * 8 + g];
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt) bb[nt] = S[(ks * 4 + q) * lds + nt * 8 + g];
-#pragma unroll
-      for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 2; ++nt) dmma(r[mt][nt], a[mt], bb[nt]);
-    }
-#pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-      for (int nt = 0; nt < 2; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-          INV[(nt * 8 + 2 * q + h) * ldi + 16 + mt * 8 + g] = -r[mt][nt][h];
-  }
-  __syncwarp();
-}
-
 // One warp: POTF2 of the nb x nb (nb <= 32) lower block at T (T[c*ldt + r]), written back
 // to T and to global (Ag, lda) — lower part, on failure up to the failing column (incl. the
 // pivot). Blocked 16 + 16: POTF2 of columns 0..15 with all 32 rows in registers (which also
