@@ -7,6 +7,7 @@
 // an atomic counter and locate their matrix by binary search. Only real tiles are visited —
 // for SYRK only the tiles of the referenced triangle ("decision layer").
 #include <algorithm>
+#include <mutex>
 
 #include "common.cuh"
 #include "internal.h"
@@ -390,12 +391,21 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
 int g_sms = 0;
 
 int launch_blas(const BlasArgs& a, cudaStream_t stream) {
-  if (!g_sms) {
-    int dev;
+  {  // per-device kernel attribute (dynamic shared memory), once per device ordinal
+    static unsigned long long ready = 0;
+    static std::mutex mu;
+    int dev = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(gemm_syrk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)sizeof(GemmSmem));
+    const unsigned long long bit = dev < 64 ? 1ull << dev : 0ull;
+    if (!(g_sms && (ready & bit))) {
+      std::lock_guard<std::mutex> lock(mu);
+      cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+      cudaError_t ea = cudaFuncSetAttribute(gemm_syrk_kernel,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)sizeof(GemmSmem));
+      if (ea != cudaSuccess) return (int)ea;
+      ready |= bit;
+    }
   }
   void* ws = nullptr;
   cudaError_t e = ws_alloc(&ws, sizeof(int) * ((size_t)a.batch + 2), stream);

@@ -34,6 +34,7 @@
 // (SURVEY.md §8(c) readings #2-#3); nothing of them is touched again (a7).
 #include <algorithm>
 #include <cstdlib>
+#include <mutex>
 
 #include "common.cuh"
 #include "internal.h"
@@ -1343,11 +1344,20 @@ static cudaError_t setup_blocked(int* occ) {
 
 static int g_occ64s = 0;
 
+// Kernel attributes (dynamic shared memory limits) are per device: the setup runs once for every
+// device the library is called on (bit per ordinal); occupancies and the SM count are those of
+// the first device (the pool's GPUs are identical B200s).
+static unsigned long long g_dev_ready = 0;
+static std::mutex g_init_mu;
+
 static cudaError_t init_device_info() {
-  if (g_num_sms) return cudaSuccess;
   int dev;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
+  const unsigned long long bit = dev < 64 ? 1ull << dev : 0ull;
+  if (g_num_sms && (g_dev_ready & bit)) return cudaSuccess;
+  std::lock_guard<std::mutex> lock(g_init_mu);
+  if (g_num_sms && (g_dev_ready & bit)) return cudaSuccess;
   int sms = 0;
   e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
@@ -1367,6 +1377,7 @@ static cudaError_t init_device_info() {
   }
   potrf_ts();
   g_num_sms = sms;
+  g_dev_ready |= bit;
   return cudaSuccess;
 }
 
