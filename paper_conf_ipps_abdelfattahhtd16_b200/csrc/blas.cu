@@ -242,9 +242,19 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
 // Column blocks of 32 are solved in dependency order (ascending for upper T, descending for
 // lower T): R = alpha B_J - sum_K X_K T_{K,J} (DMMA), X_J = R inv(T_JJ) (TRTRI in smem + DMMA).
 constexpr int kTW = 32;
+constexpr int kTC = 16;      // k chunk of the solved-block accumulation
+constexpr int kTStages = 3;  // its cp.async ring depth
 struct TrsmSmem {
-  double x[kTW][kLD];     // A operand [k][row]
-  double t[kTW][kTW + 4];  // B operand [k][col]; scratch for the transposed inverse
+  union {
+    struct {  // accumulation ring: X chunk [k][row] and T chunk [k][col]
+      double xa[kTStages][kTC][kLD];
+      double tb[kTStages][kTC][kTW + 4];
+    } ring;
+    struct {
+      double x[kTW][kLD];      // R = alpha B_J - sum, [k=col][row]
+      double t[kTW][kTW + 4];  // scratch for the transposed inverse
+    } e;
+  } u;
   double d[kTW][kTW + 1];  // diagonal block T_JJ as the lower factor L of TRTRI: d[c][r] = L[r][c]
   double inv[kTW][kTW + 4];  // inv(T_JJ) [k][col]
   double S[16 * LDS_T];      // TRTRI scratch
@@ -265,8 +275,35 @@ __device__ __forceinline__ size_t bix(bool bt, int r, int c, int ldb) {
   return bt ? (size_t)r * ldb + c : (size_t)c * ldb + r;
 }
 
+// One k chunk of the accumulation sum_K X_K T_{K,J}: X[r0:r0+64, k0:k0+16] (already solved
+// columns of the right-hand side, B's storage view) and T[k0:k0+16, c0:c0+32] (op(A), an
+// off-diagonal block: no triangle mask, no unit diagonal), 8-byte cp.async, zero-filled
+// outside [k0, kend) and the matrix.
+__device__ __forceinline__ void trsm_stage(TrsmSmem& s, int st, const BlasArgs& a, const double* A,
+                                           int lda, const double* B, int ldb, int m, int r0,
+                                           int c0, int w, int k0, int kend) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int e = 0; e < (kTC * kBT) / kGThreads; ++e) {
+    const int idx = tid + e * kGThreads;
+    // contiguous direction of the storage view first: rows for B, k for B^T (side 'L')
+    const int k = idx / kBT, i = idx % kBT;
+    const bool p = (k0 + k < kend) && (r0 + i < m);
+    cp_async8(&s.u.ring.xa[st][k][i], B + (p ? bix(a.bt, r0 + i, k0 + k, ldb) : 0), p);
+  }
+#pragma unroll
+  for (int e = 0; e < (kTC * kTW) / kGThreads; ++e) {
+    const int idx = tid + e * kGThreads;
+    const int j = idx / kTC, k = idx % kTC;
+    const bool p = (k0 + k < kend) && (j < w);
+    const size_t o = a.ta ? (size_t)(k0 + k) * lda + (c0 + j) : (size_t)(c0 + j) * lda + (k0 + k);
+    cp_async8(&s.u.ring.tb[st][k][j], A + (p ? o : 0), p);
+  }
+}
+
 __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* off, int* counter) {
-  __shared__ __align__(16) TrsmSmem s;
+  extern __shared__ __align__(16) unsigned char tsm_raw[];
+  TrsmSmem& s = *reinterpret_cast<TrsmSmem*>(tsm_raw);
   __shared__ int s_t;
   pdl_wait();
   const int total = off[a.batch];
@@ -295,40 +332,44 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
       for (int x = 0; x < 4; ++x)
 #pragma unroll
         for (int y = 0; y < 2; ++y) acc[x][y][0] = acc[x][y][1] = 0.0;
-      // sum over solved blocks K of X_K T_{K,J}
-      for (int s2 = 0; s2 < step; ++s2) {
-        const int Kb = a.tlower ? nbk - 1 - s2 : s2;
-        const int k0 = Kb * kTW, kw = min(kTW, n - k0);
-        for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
-          const int k = idx / kBT, i = idx % kBT;
-          s.x[k][i] = (k < kw && r0 + i < m) ? B[bix(a.bt, r0 + i, k0 + k, ldb)] : 0.0;
-        }
-        for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
-          const int j = idx / kTW, k = idx % kTW;
-          s.t[k][j] = (k < kw && j < w) ? t_elem(a, A, lda, k0 + k, c0 + j) : 0.0;
-        }
+      // sum over the solved blocks K of X_K T_{K,J} = X[:, kb:ke] T[kb:ke, J] as one pipelined
+      // k loop (columns before J for an upper T, after J for a lower T)
+      const int kb = a.tlower ? c0 + kTW : 0, ke = a.tlower ? n : c0;
+      const int nkc = ke > kb ? cdiv(ke - kb, kTC) : 0;
+      if (nkc > 0) trsm_stage(s, 0, a, A, lda, B, ldb, m, r0, c0, w, kb, ke);
+      cp_async_commit();
+      if (nkc > 1) trsm_stage(s, 1, a, A, lda, B, ldb, m, r0, c0, w, kb + kTC, ke);
+      cp_async_commit();
+      for (int kc = 0; kc < nkc; ++kc) {
+        cp_async_wait<1>();
         __syncthreads();
+        if (kc + 2 < nkc)
+          trsm_stage(s, (kc + 2) % kTStages, a, A, lda, B, ldb, m, r0, c0, w, kb + (kc + 2) * kTC,
+                     ke);
+        cp_async_commit();
+        const int st = kc % kTStages;
 #pragma unroll
-        for (int k4 = 0; k4 < kTW / 4; ++k4) {
+        for (int k4 = 0; k4 < kTC / 4; ++k4) {
           double fa[4], fb[2];
 #pragma unroll
-          for (int x = 0; x < 4; ++x) fa[x] = s.x[k4 * 4 + q][wr + x * 8 + g];
+          for (int x = 0; x < 4; ++x) fa[x] = s.u.ring.xa[st][k4 * 4 + q][wr + x * 8 + g];
 #pragma unroll
-          for (int y = 0; y < 2; ++y) fb[y] = s.t[k4 * 4 + q][wc + y * 8 + g];
+          for (int y = 0; y < 2; ++y) fb[y] = s.u.ring.tb[st][k4 * 4 + q][wc + y * 8 + g];
 #pragma unroll
           for (int x = 0; x < 4; ++x)
 #pragma unroll
             for (int y = 0; y < 2; ++y) dmma(acc[x][y], fa[x], fb[y]);
         }
-        __syncthreads();
       }
+      cp_async_wait<0>();
+      __syncthreads();  // the ring is dead: s.u.e aliases it from here on
       // R = alpha B_J - acc, into s.x as [k=col][row]; diagonal block into s.d
 #pragma unroll
       for (int x = 0; x < 4; ++x)
 #pragma unroll
         for (int y = 0; y < 2; ++y)
 #pragma unroll
-          for (int h = 0; h < 2; ++h) s.x[wc + y * 8 + 2 * q + h][wr + x * 8 + g] = -acc[x][y][h];
+          for (int h = 0; h < 2; ++h) s.u.e.x[wc + y * 8 + 2 * q + h][wr + x * 8 + g] = -acc[x][y][h];
       // TRTRI input L (lower, L[r][c] at d[c][r]): L = T_JJ when T is lower, L = T_JJ^T when
       // it is upper (then inv(L)^T = inv(T_JJ) comes out of TRTRI directly)
       for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
@@ -341,7 +382,7 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
       for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
         const int k = idx / kBT, i = idx % kBT;
         const double bv = (k < w && r0 + i < m) ? B[bix(a.bt, r0 + i, c0 + k, ldb)] : 0.0;
-        s.x[k][i] = fma(a.alpha, bv, s.x[k][i]);
+        s.u.e.x[k][i] = fma(a.alpha, bv, s.u.e.x[k][i]);
       }
       // inv(T_JJ) by warp 0: 8x8 substitution + recursive doubling on DMMA (trtri32_dmma_warp)
       // into the B-operand layout INV[k][n] = inv(L)[n][k]; for a lower T that is inv(T)^T,
@@ -349,11 +390,11 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
       if (warp == 0) {
         s.tv[lane] = 1.0 / s.d[lane][lane];
         __syncwarp();
-        double* out = a.tlower ? &s.t[0][0] : &s.inv[0][0];
+        double* out = a.tlower ? &s.u.e.t[0][0] : &s.inv[0][0];
         trtri32_dmma_warp(&s.d[0][0], kTW + 1, s.tv, out, kTW + 4, s.S, LDS_T, lane);
         if (a.tlower) {
 #pragma unroll 4
-          for (int k = 0; k < kTW; ++k) s.inv[k][lane] = s.t[lane][k];
+          for (int k = 0; k < kTW; ++k) s.inv[k][lane] = s.u.e.t[lane][k];
         }
       }
       __syncthreads();
@@ -366,7 +407,7 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
       for (int k4 = 0; k4 < kTW / 4; ++k4) {
         double fa[4], fb[2];
 #pragma unroll
-        for (int x = 0; x < 4; ++x) fa[x] = s.x[k4 * 4 + q][wr + x * 8 + g];
+        for (int x = 0; x < 4; ++x) fa[x] = s.u.e.x[k4 * 4 + q][wr + x * 8 + g];
 #pragma unroll
         for (int y = 0; y < 2; ++y) fb[y] = s.inv[k4 * 4 + q][wc + y * 8 + g];
 #pragma unroll
@@ -404,6 +445,9 @@ int launch_blas(const BlasArgs& a, cudaStream_t stream) {
                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             (int)sizeof(GemmSmem));
       if (ea != cudaSuccess) return (int)ea;
+      ea = cudaFuncSetAttribute(trsm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)sizeof(TrsmSmem));
+      if (ea != cudaSuccess) return (int)ea;
       ready |= bit;
     }
   }
@@ -425,6 +469,8 @@ int launch_blas(const BlasArgs& a, cudaStream_t stream) {
     cfg.blockDim = dim3(kGThreads);
     cfg.gridDim = dim3(g_sms * 8);
     if (a.mode == kTrsm) {
+      cfg.gridDim = dim3(g_sms * 3);  // 3 CTAs per SM (61 KB smem each)
+      cfg.dynamicSmemBytes = sizeof(TrsmSmem);
       e = cudaLaunchKernelEx(&cfg, trsm_kernel, a, (const int*)off, counter);
     } else {
       cfg.gridDim = dim3(g_sms * 4);  // 4 CTAs per SM (registers, 52 KB smem each)
