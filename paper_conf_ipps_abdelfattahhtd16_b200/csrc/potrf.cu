@@ -988,6 +988,74 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
 //                   overwrites s.inv with inv(L11) of panel p+1 (single inverse buffer).
 // Arrivals and syncs are paired under the same conditions (panel p has blocks below it and
 // did not fail), so no barrier phase is left open across matrices.
+// One matrix by a (diagonal warp, off-diagonal warp) pair; named barriers bar0 (ready),
+// bar0+1 (block 1 stored), bar0+2 (inverse free).
+template <bool UP, typename E>
+VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, int n, int ld,
+                         int* info_out, int bar0) {
+  const int g = lane >> 2, q = lane & 3;
+  const int npan = (n + 31) / 32;
+  if (role == 0) {
+    bool pending_free = false;  // the other warp will arrive inv_free for the previous panel
+    for (int p = 0; p < npan; ++p) {
+      const int j0 = 32 * p, nb = min(32, n - j0);
+      const bool below = p + 1 < npan;
+      double acc[4][4][2];
+      small_acc_init<UP, E>(acc, A, n, ld, j0, j0, nb, true, lane);
+      if (p > 0) {
+        // columns of the panels before p-1 are final: their update runs while the other warp
+        // is still on block 1 of panel p-1; the newest 32 columns after block 1 is stored
+        small_kloop<UP, E>(acc, A, n, ld, j0, j0, 0, j0 - 32, lane);
+        bar_group(bar0 + 1, 64);  // block 1 of panel p-1 (= these rows) is stored
+        small_kloop<UP, E>(acc, A, n, ld, j0, j0, j0 - 32, j0, lane);
+      }
+#pragma unroll
+      for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+          s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+          s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+        }
+      __syncwarp();
+      const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
+                                         s.wbuf, s.sv, s.tv);
+      if (pending_free) {  // the other warp is done with inv(L11) of panel p-1
+        bar_group(bar0 + 2, 64);
+        pending_free = false;
+      }
+      if (info) {
+        if (lane == 0) {
+          s.info = info;
+          *info_out = j0 + info;
+        }
+        if (below) bar_group_arrive(bar0, 64);  // the other warp reads s.info and stops
+        break;
+      }
+      if (!below) break;
+      trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
+      if (lane == 0) s.info = 0;
+      bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready
+      pending_free = true;
+    }
+  } else {
+    for (int p = 0; p + 1 < npan; ++p) {  // panels with blocks below the diagonal
+      const int j0 = 32 * p;
+      const int nblk = (n - j0 + 31) / 32;
+      double acc[4][4][2];
+      small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
+      bar_group(bar0, 64);  // inv(L11) of panel p (or the failure)
+      if (s.info) break;
+      small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane);
+      bar_group_arrive(bar0 + 1, 64);  // block 1 stored: the diagonal warp may start panel p+1
+      for (int b = 2; b < nblk; ++b) {
+        small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
+        small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
+      }
+      bar_group_arrive(bar0 + 2, 64);  // done with s.inv of panel p
+    }
+  }
+}
+
 template <bool UP, typename E = double>
 __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     potrf_small_la_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
@@ -1001,7 +1069,6 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
   const int count = *(volatile const int*)&ctrl->count[range];
   const int start = *(volatile const int*)&ctrl->start[range];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int g = lane >> 2, q = lane & 3;
   for (;;) {
     if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
     __syncthreads();
@@ -1009,72 +1076,47 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     __syncthreads();
     if (it >= count) break;
     const int m = order[start + it];
-    const int n = d_n[m], ld = d_ldda[m];
-    E* A = dA[m];
     TL_BEGIN(t_tl)
-    const int npan = (n + 31) / 32;
-    if (warp == 0) {
-      bool pending_free = false;  // warp 1 will arrive inv_free for the previous panel
-      for (int p = 0; p < npan; ++p) {
-        const int j0 = 32 * p, nb = min(32, n - j0);
-        const bool below = p + 1 < npan;
-        double acc[4][4][2];
-        small_acc_init<UP, E>(acc, A, n, ld, j0, j0, nb, true, lane);
-        if (p > 0) {
-          // columns of the panels before p-1 are final: their update runs while warp 1 is
-          // still on block 1 of panel p-1; the newest 32 columns after block 1 is stored
-          small_kloop<UP, E>(acc, A, n, ld, j0, j0, 0, j0 - 32, lane);
-          bar_group(2, 64);  // block 1 of panel p-1 (= these rows) is stored
-          small_kloop<UP, E>(acc, A, n, ld, j0, j0, j0 - 32, j0, lane);
-        }
-#pragma unroll
-        for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-          for (int nt = 0; nt < 4; ++nt) {
-            s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
-            s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
-          }
-        __syncwarp();
-        const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
-                                           s.wbuf, s.sv, s.tv);
-        if (pending_free) {  // warp 1 is done with inv(L11) of panel p-1
-          bar_group(3, 64);
-          pending_free = false;
-        }
-        if (info) {
-          if (lane == 0) {
-            s.info = info;
-            d_info[m] = j0 + info;
-          }
-          if (below) bar_group_arrive(1, 64);  // warp 1 reads s.info and stops
-          break;
-        }
-        if (!below) break;
-        trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
-        if (lane == 0) s.info = 0;
-        bar_group_arrive(1, 64);  // inv(L11) of panel p is ready
-        pending_free = true;
-      }
-    } else {
-      for (int p = 0; p + 1 < npan; ++p) {  // panels with blocks below the diagonal
-        const int j0 = 32 * p;
-        const int nblk = (n - j0 + 31) / 32;
-        double acc[4][4][2];
-        small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
-        bar_group(1, 64);  // inv(L11) of panel p (or the failure)
-        if (s.info) break;
-        small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane);
-        bar_group_arrive(2, 64);  // block 1 stored: warp 0 may start panel p+1
-        for (int b = 2; b < nblk; ++b) {
-          small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
-          small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
-        }
-        bar_group_arrive(3, 64);  // done with s.inv of panel p
-      }
-    }
+    la_matrix<UP, E>(s, warp, lane, dA[m], d_n[m], d_ldda[m], d_info + m, 1);
     __syncthreads();
     if (tid == 0) s.info = 0;
     TL_END(tid == 0, t_tl, m, 21)
+  }
+}
+
+// The same pairs packed two per 4-warp CTA with the roles on fixed sub-partitions: warps 0/1 are
+// the diagonal warps of pair 0/1, warps 2/3 their off-diagonal warps (warp w runs on SMSP
+// w % 4), so the pivot chains share their sub-partitions only with other pivot chains, not
+// with the off-diagonal DMMA streams (tools/contention_bench.cu: a DMMA stream starves the
+// FP64 chain on its sub-partition). Each pair fetches its own matrices.
+template <bool UP, typename E = double>
+__global__ void __launch_bounds__(128, 4)
+    potrf_small_la2_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
+                           const int* __restrict__ d_ldda, int* __restrict__ d_info,
+                           const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
+                           int range, int wait_upstream) {
+  __shared__ SmallSmem ss[2];
+  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
+  if (wait_upstream) pdl_wait();
+  pdl_launch_dependents();
+  const int count = *(volatile const int*)&ctrl->count[range];
+  const int start = *(volatile const int*)&ctrl->start[range];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int pair = warp & 1, role = warp >> 1;
+  SmallSmem& s = ss[pair];
+  const int bar0 = 1 + 4 * pair, tsync = 4 + 4 * pair;
+  for (;;) {
+    if (role == 0 && lane == 0) s.item = atomicAdd(&ctrl->head[range], 1);
+    bar_group(tsync, 64);
+    const int it = s.item;
+    bar_group(tsync, 64);
+    if (it >= count) break;
+    const int m = order[start + it];
+    TL_BEGIN(t_tl)
+    la_matrix<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
+    bar_group(tsync, 64);
+    if (role == 0 && lane == 0) s.info = 0;
+    TL_END(role == 0 && lane == 0, t_tl, m, 22)
   }
 }
 
@@ -1373,7 +1415,7 @@ static cudaError_t init_device_info() {
   if (g_occ_wsmall < 1) g_occ_wsmall = 1;
   {
     const char* v = getenv("VB_SMALL");
-    g_small = v ? atoi(v) : 3;
+    g_small = v ? atoi(v) : 4;
   }
   potrf_ts();
   g_num_sms = sms;
@@ -1426,7 +1468,12 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
     cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
     cfg.dynamicSmemBytes = 0;
     if constexpr (sizeof(E) == 8) {
-      if (g_small == 3) {
+      if (g_small == 4) {
+        cfg.blockDim = dim3(128);
+        cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
+        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true> : potrf_small_la2_kernel<false>,
+                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
+      } else if (g_small == 3) {
         e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true> : potrf_small_la_kernel<false>,
                                d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
       } else if (g_small == 2) {
@@ -1439,7 +1486,9 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
                                d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
       }
     } else {
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true, E> : potrf_small_la_kernel<false, E>,
+      cfg.blockDim = dim3(128);
+      cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, E> : potrf_small_la2_kernel<false, E>,
                              d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
     }
     if (e != cudaSuccess) return e;
