@@ -7,7 +7,7 @@ functions raises.
 
 Arguments that the C ABI takes as device pointers accept either an int (raw address) or a
 torch CUDA tensor of the right dtype (int32 for sizes/info, int64 for pointer arrays,
-float64 for matrices). ``stream`` accepts None (torch's current stream), a
+float64 for matrices, float32 for vbatched_spotrf). ``stream`` accepts None (torch's current stream), a
 ``torch.cuda.Stream`` or a raw handle.
 """
 from __future__ import annotations
