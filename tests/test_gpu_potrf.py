@@ -349,22 +349,23 @@ def test_stream_semantics():
     assert torch.equal(db.arena, ref.arena)  # deterministic across streams / runs
 
 
-def test_host_api_chunked():
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_host_api_chunked(uplo):
     """vbatched_dpotrf_host: host buffers, small workspace -> many chunks; bit-identical to the
-    device API on the same inputs."""
+    device API on the same inputs (both storage triangles)."""
     from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dpotrf_host
     n = vbgen.sizes("C3")[:400]
-    dev = DeviceBatch(n, seed=3).fill()
+    dev = DeviceBatch(n, seed=3, nonspd_mod=20).fill(poison=True, uplo=uplo)
     torch.cuda.synchronize()
     host = dev.arena.cpu().numpy().copy()
-    dev.dpotrf()
+    dev.dpotrf(uplo=uplo)
     torch.cuda.synchronize()
     ptrs = (host.ctypes.data + 8 * dev.off).astype(np.int64)
     info = np.full(dev.B, -99, dtype=np.int32)
-    vbatched_dpotrf_host("L", dev.n, ptrs, dev.ldda, info, dev.B, int(n.max()),
+    vbatched_dpotrf_host(uplo, dev.n, ptrs, dev.ldda, info, dev.B, int(n.max()),
                          workspace_bytes=3 * 48 << 20)
-    assert np.array_equal(info, dev.info())
-    assert np.array_equal(host, dev.arena.cpu().numpy())
+    assert np.array_equal(info, dev.info()) and (info > 0).sum() == 20
+    assert np.array_equal(host.view(np.uint64), dev.arena.cpu().numpy().view(np.uint64))
 
 
 @pytest.mark.parametrize("cfg", ["C3", "C4"])
