@@ -46,11 +46,14 @@ namespace vb {
 #ifdef VB_PHASE_PROF
 __device__ unsigned long long g_phase[8];
 #define VB_T0(v) long long v = clock64();
+#define VB_ADDW(i, v) \
+  if ((threadIdx.x & 31) == 0) atomicAdd(&g_phase[i], (unsigned long long)(clock64() - (v)));
 #define VB_ADD(i, v) \
   if (threadIdx.x == 0) atomicAdd(&g_phase[i], (unsigned long long)(clock64() - (v)));
 #else
 #define VB_T0(v)
 #define VB_ADD(i, v)
+#define VB_ADDW(i, v)
 #endif
 // Diagonal-block step timers (tools/diag_bench.cu built with -DVB_DIAG_PROF): thread 0
 // accumulates clock64() deltas between consecutive marks into g_dprof[i].
@@ -863,7 +866,8 @@ VB_DEVINL void small_panel_update(double (&acc)[4][4][2], const E* __restrict__ 
 // skipped), then direct stores of rows < n.
 template <bool UP, typename E = double>
 VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], E* __restrict__ A,
-                                int n, int ld, int r0, int j0, int lane) {
+                                int n, int ld, int r0, int j0, int lane,
+                                double (*xs)[36] = nullptr) {
   const int g = lane >> 2, q = lane & 3;
   double x[4][4][2];
 #pragma unroll
@@ -892,6 +896,8 @@ VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], E* __restr
       for (int h = 0; h < 2; ++h) {
         const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
         if (row < n) A[gix<UP>(row, j0 + col, ld)] = x[mt][nt][h];
+        // optional copy for the next diagonal update, as stored (rounded to E), [col][row]
+        if (xs) xs[col][mt * 8 + g] = row < n ? (double)(E)x[mt][nt][h] : 0.0;
       }
 }
 
@@ -1001,13 +1007,34 @@ VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, in
       const int j0 = 32 * p, nb = min(32, n - j0);
       const bool below = p + 1 < npan;
       double acc[4][4][2];
+      VB_T0(t0)
       small_acc_init<UP, E>(acc, A, n, ld, j0, j0, nb, true, lane);
       if (p > 0) {
         // columns of the panels before p-1 are final: their update runs while the other warp
         // is still on block 1 of panel p-1; the newest 32 columns after block 1 is stored
         small_kloop<UP, E>(acc, A, n, ld, j0, j0, 0, j0 - 32, lane);
+        VB_ADDW(0, t0)
+        VB_T0(t1)
         bar_group(bar0 + 1, 64);  // block 1 of panel p-1 (= these rows) is stored
-        small_kloop<UP, E>(acc, A, n, ld, j0, j0, j0 - 32, j0, lane);
+        VB_ADDW(1, t1)
+        VB_T0(t2)
+        // the newest 32 columns: block 1 of panel p-1, which the other warp also left in s.T
+        // ([col][row], the stored values): a SYRK from shared memory instead of L2, same k order
+#pragma unroll
+        for (int ks = 0; ks < 8; ++ks) {
+          double fa[4], fb[4];
+#pragma unroll
+          for (int t = 0; t < 4; ++t) {
+            fb[t] = s.T[ks * 4 + q][t * 8 + g];
+            fa[t] = -fb[t];
+          }
+#pragma unroll
+          for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+        }
+        __syncwarp();  // all reads of s.T done before it is overwritten with the tile
+        VB_ADDW(2, t2)
       }
 #pragma unroll
       for (int mt = 0; mt < 4; ++mt)
@@ -1017,8 +1044,11 @@ VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, in
           s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
         }
       __syncwarp();
+      VB_T0(t3)
       const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
                                          s.wbuf, s.sv, s.tv);
+      VB_ADDW(3, t3)
+      VB_T0(t4)
       if (pending_free) {  // the other warp is done with inv(L11) of panel p-1
         bar_group(bar0 + 2, 64);
         pending_free = false;
@@ -1035,6 +1065,7 @@ VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, in
       trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
       if (lane == 0) s.info = 0;
       bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready
+      VB_ADDW(4, t4)
       pending_free = true;
     }
   } else {
@@ -1042,14 +1073,27 @@ VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, in
       const int j0 = 32 * p;
       const int nblk = (n - j0 + 31) / 32;
       double acc[4][4][2];
+      VB_T0(t5)
       small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
+      VB_ADDW(5, t5)
+      VB_T0(t6)
       bar_group(bar0, 64);  // inv(L11) of panel p (or the failure)
+      VB_ADDW(6, t6)
       if (s.info) break;
-      small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane);
+      VB_T0(t7)
+      // block 1 = the rows of the next diagonal block: also leave it in s.T (free since the
+      // diagonal warp finished TRTRI(p); it reads it after the block1 barrier)
+      small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane, s.T);
+      __syncwarp();
+      VB_ADDW(7, t7)
       bar_group_arrive(bar0 + 1, 64);  // block 1 stored: the diagonal warp may start panel p+1
       for (int b = 2; b < nblk; ++b) {
+        VB_T0(t8)
         small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
+        VB_ADDW(5, t8)
+        VB_T0(t9)
         small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
+        VB_ADDW(7, t9)
       }
       bar_group_arrive(bar0 + 2, 64);  // done with s.inv of panel p
     }
