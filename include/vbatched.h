@@ -76,6 +76,9 @@ int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const in
  * cp.async staging path instead of TMA bulk copies. */
 int vbatched_spotrf(char uplo, const int* d_n, float* const* dA_array, const int* d_ldda,
                     int* d_info, int batchCount, int max_n, vb_stream_t stream);
+/* FP32 LAPACK-like interface (no max_n; see vbatched_dpotrf_nomax). */
+int vbatched_spotrf_nomax(char uplo, const int* d_n, float* const* dA_array, const int* d_ldda,
+                          int* d_info, int batchCount, vb_stream_t stream);
 
 /* LAPACK-like interface: identical to vbatched_dpotrf but max_n is not
  * needed; the device scan computes it (no host synchronisation: launch sizes assume the

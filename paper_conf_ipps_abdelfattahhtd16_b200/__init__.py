@@ -48,6 +48,7 @@ def lib() -> ctypes.CDLL:
         L.vbatched_dpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
         L.vbatched_dpotrf_nomax.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _vp]
         L.vbatched_spotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
+        L.vbatched_spotrf_nomax.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _vp]
         L.vbatched_dpotrf_workspace_size.argtypes = [_i]
         L.vbatched_dpotrf_workspace_size.restype = ctypes.c_size_t
         L.vbatched_dpotrf_scan.argtypes = [_c, _vp, _vp, _vp, _i, _i, _vp, _vp]
@@ -68,7 +69,7 @@ def lib() -> ctypes.CDLL:
         L.vbatched_host_alloc.restype = _vp
         L.vbatched_host_free.argtypes = [_vp]
         for name in ("vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
-                     "vbatched_spotrf",
+                     "vbatched_spotrf", "vbatched_spotrf_nomax",
                      "vbatched_dpotrf_scan", "vbatched_dpotrf_factor",
                      "vbatched_dgemm", "vbatched_dsyrk", "vbatched_dtrsm",
                      "vbatched_dpotrs", "vbatched_dposv",
@@ -120,6 +121,12 @@ def vbatched_spotrf(uplo, n, dA_array, ldda, info, batchCount, max_n, stream=Non
     rc = lib().vbatched_spotrf(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
                                int(batchCount), int(max_n), _stream(stream))
     return _check(rc, "vbatched_spotrf") if check else rc
+
+
+def vbatched_spotrf_nomax(uplo, n, dA_array, ldda, info, batchCount, stream=None, check=True):
+    rc = lib().vbatched_spotrf_nomax(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
+                                     int(batchCount), _stream(stream))
+    return _check(rc, "vbatched_spotrf_nomax") if check else rc
 
 
 def vbatched_dpotrf_nomax(uplo, n, dA_array, ldda, info, batchCount, stream=None, check=True):

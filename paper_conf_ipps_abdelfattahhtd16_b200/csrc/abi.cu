@@ -99,6 +99,12 @@ int vbatched_spotrf(char uplo, const int* d_n, float* const* dA_array, const int
                     (cudaStream_t)stream);
 }
 
+int vbatched_spotrf_nomax(char uplo, const int* d_n, float* const* dA_array, const int* d_ldda,
+                          int* d_info, int batchCount, vb_stream_t stream) {
+  return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, 0, false,
+                    (cudaStream_t)stream);
+}
+
 int vbatched_dpotrf_nomax(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
                           int* d_info, int batchCount, vb_stream_t stream) {
   return potrf_impl(uplo, d_n, dA_array, d_ldda, d_info, batchCount, 0, false,

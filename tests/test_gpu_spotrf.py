@@ -80,3 +80,18 @@ def test_spotrf_exact_family():
     assert np.all(db.info() == 0)
     for i, ni in enumerate(sizes):
         assert np.array_equal(np.tril(db.block(i)[:ni, :ni]), np.tril(np.ones((ni, ni), np.float32)))
+
+
+def test_spotrf_nomax_equals_max_given():
+    import paper_conf_ipps_abdelfattahhtd16_b200 as vb
+    n = vbgen.sizes("C3")[:300]
+    a = DeviceBatch(n, seed=3, nonspd_mod=20, dtype="f32").fill(poison=True)
+    b = DeviceBatch(n, seed=3, nonspd_mod=20, dtype="f32").fill(poison=True)
+    a.dpotrf()
+    vb.vbatched_spotrf_nomax("L", b.d_n, b.d_ptrs, b.d_ldda, b.d_info, b.B)
+    torch.cuda.synchronize()
+    assert np.array_equal(a.info(), b.info())
+    ha, hb = a.arena.cpu().numpy(), b.arena.cpu().numpy()
+    for i in range(a.B):  # the matrices' blocks (the arenas' alignment gaps are never written)
+        sl = slice(int(a.off[i]), int(a.off[i]) + int(a.ldda[i]) * max(int(n[i]), 0))
+        assert np.array_equal(ha[sl].view(np.uint32), hb[sl].view(np.uint32)), i
