@@ -452,3 +452,40 @@ def test_uplo_upper_device_generated_c3_sample():
         assert np.array_equal(bl[:k, :k].view(np.uint64)[low], bu[:k, :k].T.view(np.uint64)[low]), i
         strict_low = np.tril(np.ones((ni, ni), bool), -1)
         assert np.all(bu[:ni, :ni].view(np.uint64)[strict_low] == POISON), i
+
+
+@pytest.mark.parametrize("uplo", ["L", "U"])
+def test_two_phase_api_equals_single_call(uplo):
+    """vbatched_dpotrf_scan + vbatched_dpotrf_factor on caller workspace (the split bench.py's
+    roofline pass times) give exactly the single call's result, both storage triangles."""
+    import paper_conf_ipps_abdelfattahhtd16_b200 as vb
+    n = vbgen.sizes("C4")[:500]
+    a = DeviceBatch(n, seed=4, nonspd_mod=20).fill(poison=True, uplo=uplo)
+    b = DeviceBatch(n, seed=4, nonspd_mod=20).fill(poison=True, uplo=uplo)
+    mx = int(n.max())
+    a.dpotrf(uplo=uplo)
+    ws = torch.empty(vb.vbatched_dpotrf_workspace_size(b.B), dtype=torch.uint8, device="cuda")
+    vb.vbatched_dpotrf_scan(uplo, b.d_n, b.d_ldda, b.d_info, b.B, mx, ws)
+    vb.vbatched_dpotrf_factor(uplo, b.d_n, b.d_ptrs, b.d_ldda, b.d_info, b.B, mx, ws)
+    torch.cuda.synchronize()
+    assert np.array_equal(a.info(), b.info()) and (a.info() > 0).sum() == 25
+    ha, hb = a.arena.cpu().numpy(), b.arena.cpu().numpy()
+    for i in range(a.B):
+        sl = slice(int(a.off[i]), int(a.off[i]) + int(a.ldda[i]) * int(n[i]))
+        assert np.array_equal(ha[sl].view(np.uint64), hb[sl].view(np.uint64)), i
+
+
+def test_max_n_too_small_f32_and_upper():
+    """n > max_n -> info -7 and the matrix untouched, for SPOTRF and for uplo 'U' too."""
+    n = np.array([40, 300, 100, 700], dtype=np.int32)
+    for dtype, uplo in (("f32", "L"), ("f64", "U")):
+        db = DeviceBatch(n, seed=6, dtype=dtype).fill(poison=True, uplo=uplo)
+        before = db.arena.cpu().numpy().copy()
+        db.dpotrf(max_n=200, uplo=uplo)
+        torch.cuda.synchronize()
+        info = db.info()
+        assert list(info[[1, 3]]) == [-7, -7] and list(info[[0, 2]]) == [0, 0], (dtype, uplo, info)
+        after = db.arena.cpu().numpy()
+        for i in (1, 3):
+            sl = slice(int(db.off[i]), int(db.off[i]) + int(db.ldda[i]) * int(n[i]))
+            assert np.array_equal(before[sl], after[sl], equal_nan=True), (dtype, uplo, i)
