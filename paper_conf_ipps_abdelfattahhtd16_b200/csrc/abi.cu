@@ -256,8 +256,9 @@ const char* vbatched_version(void) {
   if (cudaGetDeviceCount(&dev_count) == cudaSuccess && dev_count > 0) potrf_occupancy(occ);
   else cudaGetLastError();
   snprintf(buf, sizeof buf,
-           "libvbatched 0.5 (sm_100a; DMMA m8n8k4 f64; n>%d: blocked NB=64, %d compute warps + TMA "
-           "producer, %d CTAs/SM; 32<n<=%d: small kernel, %d CTAs/SM; n<=32: warp per matrix)",
+           "libvbatched 0.6 (sm_100a; DMMA m8n8k4 f64; n>%d: blocked NB=64, %d compute warps + TMA "
+           "producer, %d CTAs/SM; 32<n<=%d: paired look-ahead small kernel, %d CTAs/SM; n<=32: "
+           "warp per matrix; FP64 and FP32 storage, uplo L/U)",
            potrf_ts(), occ[1], occ[0], potrf_ts(), occ[3]);
   return buf;
 }

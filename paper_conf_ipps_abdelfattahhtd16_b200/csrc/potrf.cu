@@ -1563,7 +1563,7 @@ void potrf_occupancy(int* out4) {
   out4[0] = g_occ64;
   out4[1] = Cfg64d::WARPS;
   out4[2] = 0;  // (no separate NB=32 range)
-  out4[3] = g_small >= 2 ? g_occ_small : g_occ_wsmall;
+  out4[3] = g_small == 4 ? 4 : (g_small >= 2 ? g_occ_small : g_occ_wsmall);
 }
 
 int potrf_num_launches(int max_n_hint) {
