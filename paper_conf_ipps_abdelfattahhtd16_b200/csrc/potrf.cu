@@ -1100,6 +1100,104 @@ VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, in
   }
 }
 
+// Variant with the roles split by instruction mix (VB_SMALL=5): the diagonal warp runs only the
+// pivot chain (POTF2 + TRTRI of the tile in s.T); the off-diagonal warp does every DMMA update,
+// including the next diagonal tile: right after the TRSM of block 1 of panel p (the rows of the
+// next diagonal block) it leaves that block in s.T, adds the update by all older columns from
+// L2 and by block 1 itself from smem, and hands the tile over. Barriers (64 threads):
+// bar0 = inv ready (D -> O), bar0+1 = tile ready (O -> D), bar0+2 = inverse free (O -> D).
+template <bool UP, typename E>
+VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A, int n, int ld,
+                            int* info_out, int bar0) {
+  const int g = lane >> 2, q = lane & 3;
+  const int npan = (n + 31) / 32;
+  if (role == 0) {
+    bool pending_free = false;
+    for (int p = 0; p < npan; ++p) {
+      const int j0 = 32 * p, nb = min(32, n - j0);
+      const bool below = p + 1 < npan;
+      bar_group(bar0 + 1, 64);  // tile of panel p in s.T
+      const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
+                                         s.wbuf, s.sv, s.tv);
+      if (pending_free) {
+        bar_group(bar0 + 2, 64);
+        pending_free = false;
+      }
+      if (info) {
+        if (lane == 0) {
+          s.info = info;
+          *info_out = j0 + info;
+        }
+        if (below) bar_group_arrive(bar0, 64);
+        break;
+      }
+      if (!below) break;
+      trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
+      if (lane == 0) s.info = 0;
+      bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready (s.T is free again)
+      pending_free = true;
+    }
+  } else {
+    {  // tile of panel 0: A's diagonal block as it is
+      double acc[4][4][2];
+      small_acc_init<UP, E>(acc, A, n, ld, 0, 0, min(32, n), true, lane);
+#pragma unroll
+      for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+          s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+          s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+        }
+      __syncwarp();
+      bar_group_arrive(bar0 + 1, 64);
+    }
+    for (int p = 0; p + 1 < npan; ++p) {  // panels with blocks below the diagonal
+      const int j0 = 32 * p;
+      const int nblk = (n - j0 + 31) / 32;
+      double acc[4][4][2];
+      small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
+      bar_group(bar0, 64);  // inv(L11) of panel p (or the failure)
+      if (s.info) break;
+      // block 1 -> global and, as stored, into s.T ([col][row]) for the next tile's update
+      small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane, s.T);
+      __syncwarp();
+      {  // the tile of panel p+1 (rows/cols j0+32..): A - L[., 0:j0] L[., 0:j0]^T - X1 X1^T
+        const int j1 = j0 + 32, nb1 = min(32, n - j1);
+        small_acc_init<UP, E>(acc, A, n, ld, j1, j1, nb1, true, lane);
+        small_kloop<UP, E>(acc, A, n, ld, j1, j1, 0, j0, lane);
+#pragma unroll
+        for (int ks = 0; ks < 8; ++ks) {
+          double fa[4], fb[4];
+#pragma unroll
+          for (int t = 0; t < 4; ++t) {
+            fb[t] = s.T[ks * 4 + q][t * 8 + g];
+            fa[t] = -fb[t];
+          }
+#pragma unroll
+          for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < 4; ++nt) {
+            s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
+            s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
+          }
+        __syncwarp();
+        bar_group_arrive(bar0 + 1, 64);  // tile of panel p+1 ready
+      }
+      for (int b = 2; b < nblk; ++b) {
+        small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
+        small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
+      }
+      bar_group_arrive(bar0 + 2, 64);  // done with s.inv of panel p
+    }
+  }
+}
+
 template <bool UP, typename E = double>
 __global__ void __launch_bounds__(32 * kSmallWarps, 8)
     potrf_small_la_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
@@ -1133,7 +1231,7 @@ __global__ void __launch_bounds__(32 * kSmallWarps, 8)
 // w % 4), so the pivot chains share their sub-partitions only with other pivot chains, not
 // with the off-diagonal DMMA streams (tools/contention_bench.cu: a DMMA stream starves the
 // FP64 chain on its sub-partition). Each pair fetches its own matrices.
-template <bool UP, typename E = double>
+template <bool UP, typename E = double, bool SPLIT = false>
 __global__ void __launch_bounds__(128, 4)
     potrf_small_la2_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                            const int* __restrict__ d_ldda, int* __restrict__ d_info,
@@ -1157,7 +1255,10 @@ __global__ void __launch_bounds__(128, 4)
     if (it >= count) break;
     const int m = order[start + it];
     TL_BEGIN(t_tl)
-    la_matrix<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
+    if constexpr (SPLIT)
+      la_matrix_v2<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
+    else
+      la_matrix<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
     bar_group(tsync, 64);
     if (role == 0 && lane == 0) s.info = 0;
     TL_END(role == 0 && lane == 0, t_tl, m, 22)
@@ -1459,7 +1560,7 @@ static cudaError_t init_device_info() {
   if (g_occ_wsmall < 1) g_occ_wsmall = 1;
   {
     const char* v = getenv("VB_SMALL");
-    g_small = v ? atoi(v) : 4;
+    g_small = v ? atoi(v) : 5;
   }
   potrf_ts();
   g_num_sms = sms;
@@ -1512,7 +1613,13 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
     cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
     cfg.dynamicSmemBytes = 0;
     if constexpr (sizeof(E) == 8) {
-      if (g_small == 4) {
+      if (g_small == 5) {
+        cfg.blockDim = dim3(128);
+        cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
+        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, double, true>
+                                        : potrf_small_la2_kernel<false, double, true>,
+                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
+      } else if (g_small == 4) {
         cfg.blockDim = dim3(128);
         cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
         e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true> : potrf_small_la2_kernel<false>,
@@ -1532,7 +1639,8 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
     } else {
       cfg.blockDim = dim3(128);
       cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, E> : potrf_small_la2_kernel<false, E>,
+      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, E, true>
+                                      : potrf_small_la2_kernel<false, E, true>,
                              d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
     }
     if (e != cudaSuccess) return e;
@@ -1563,7 +1671,7 @@ void potrf_occupancy(int* out4) {
   out4[0] = g_occ64;
   out4[1] = Cfg64d::WARPS;
   out4[2] = 0;  // (no separate NB=32 range)
-  out4[3] = g_small == 4 ? 4 : (g_small >= 2 ? g_occ_small : g_occ_wsmall);
+  out4[3] = g_small >= 4 ? 4 : (g_small >= 2 ? g_occ_small : g_occ_wsmall);
 }
 
 int potrf_num_launches(int max_n_hint) {

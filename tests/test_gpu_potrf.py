@@ -150,7 +150,7 @@ print("OK")
     assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
 
 
-@pytest.mark.parametrize("small", ["1", "2", "3", "4"])
+@pytest.mark.parametrize("small", ["1", "2", "3", "4", "5"])
 def test_small_kernel_variants(small):
     """Both small-matrix kernels (VB_SMALL=1 warp-per-matrix, 2 = two warps per matrix) on C2
     sizes plus failing pivots in every 8-column sub-block (subprocess: the variant is read at
