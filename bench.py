@@ -63,6 +63,10 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=8.0,
                    help="target wall seconds of the bounded oracle sample")
+    p.add_argument("--clock-soak", type=float, default=1.0,
+                   help="seconds of untimed back-to-back steps run under the clock sampler right "
+                        "before the timed region (short configs: the timed region alone is too "
+                        "short for nvidia-smi to sample)")
     return p.parse_args()
 
 
@@ -81,7 +85,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={','.join(self.FIELDS)}",
-                 "--format=csv,noheader,nounits", "-lms", "100"],
+                 "--format=csv,noheader,nounits", "-lms", "20"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -321,12 +325,28 @@ def our_arm(args, cfg, rank, world, local_rank):
     barrier()
     torch.cuda.synchronize()
     sampler.start()
+    # clock soak: the same prepare+step sequence, untimed, for >= --clock-soak seconds, so that
+    # the sampler (20 ms period) sees the clocks under this load even when the K timed steps
+    # last only a few ms (C1-C4); the timed region follows immediately
+    t_soak = time.perf_counter()
+    soak_steps = 0
+    while time.perf_counter() - t_soak < args.clock_soak:
+        prepare()
+        step([torch.cuda.Event(enable_timing=True) for _ in range(2)])
+        soak_steps += 1
+        if soak_steps % 8 == 0:
+            torch.cuda.synchronize()
+    torch.cuda.synchronize()
+    barrier()
+    torch.cuda.synchronize()
     for k in range(args.steps):
         prepare()
         step(evs[k])
     torch.cuda.synchronize()
     barrier()
     clocks = sampler.stop()
+    clocks["window"] = (f"{args.clock_soak:.1f} s soak of the same steps ({soak_steps} untimed) "
+                        "immediately before the timed region + the timed region, 20 ms period")
     step_ms = [e[0].elapsed_time(e[1]) for e in evs]
     # roofline pass (after the timed region, same inputs and launch configuration): K steps
     # of the two-phase API, CUDA events around the factorisation launches
@@ -353,7 +373,7 @@ def our_arm(args, cfg, rank, world, local_rank):
         per_rank_ms = [float(x.item()) for x in allt]
     value = flops_total * args.steps / (max_total_ms / 1e3) / 1e9
 
-    # roofline of the dominant kernel (potrf_persistent_kernel) on this rank
+    # roofline of the factorisation launches (everything after the scan) on this rank
     kern_avg_s = sum(kern_ms) / args.steps / 1e3
     if cfg.nmax >= 256:
         peak, src = load_fp64_peak()
@@ -368,8 +388,9 @@ def our_arm(args, cfg, rank, world, local_rank):
     tr = load_traffic(cfg.name + ("_s" if single else ""))
     roof["traffic"] = tr.get("bytes_per_launch") if tr else None
     if tr:
-        roof["traffic_source"] = tr.get("source")
-    roof["kernel"] = "potrf_blocked3_kernel (NB=64) + potrf_small_kernel + potrf_warp_kernel (the factorisation launches)"
+        roof["traffic_source"] = ("NOT measured in this run: read from the committed ncu capture "
+                                  f"profiles/ncu_traffic_{cfg.name}.json ({tr.get('source')})")
+    roof["kernel"] = vb.factor_kernel_names(max_n)
     roof["kernel_ms"] = sum(kern_ms) / args.steps
     roof["scan_ms"] = sum(scan_ms) / args.steps
     roof["timing"] = ("kernel_ms: CUDA events around the factorisation launches in a second pass "
@@ -477,13 +498,32 @@ def e2e_leg(args, cfg, db, n_loc, max_n, world, dev):
         vb.vbatched_host_free(hp)
 
 
+def relaunch_under_torchrun(args) -> int:
+    """`python bench.py --gpus N` (N > 1) without torchrun: re-launch this command as N ranks
+    (one process per GPU) through torch.distributed.run on 127.0.0.1, so that --gpus N always
+    measures N ranks. Returns torchrun's exit code."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr=127.0.0.1", f"--master-port={port}",
+           os.path.abspath(__file__), *sys.argv[1:]]
+    log("bench: --gpus", args.gpus, "without WORLD_SIZE: re-launching as", " ".join(cmd[1:6]))
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(relaunch_under_torchrun(args))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
-        log(f"note: WORLD_SIZE={world}, --gpus={args.gpus}; using WORLD_SIZE")
+        log(f"error: WORLD_SIZE={world} but --gpus={args.gpus}: the line would report the wrong "
+            "GPU count")
+        sys.exit(2)
     cfg = vbgen.CONFIGS[args.config]
     if args.impl == "reference":
         reference_arm(args, cfg, rank, world)

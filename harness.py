@@ -104,3 +104,43 @@ def compare_with_oracle(A_in: np.ndarray, L_gpu: np.ndarray, info_gpu: int, kapp
     res["ok"] = (res["info_oracle"] == res["info_gpu"] and res["bwd"] <= 10.0 and
                  (res["rowscaled"] <= 1e-10 or not kappa_ok))
     return res
+
+
+def gpu_backward_errors(db: DeviceBatch, chunk_elems: int = 1 << 26) -> np.ndarray:
+    """Per-matrix backward error ||A - L L^T||_F / (n ||A||_F 2^-53) of every info == 0 matrix
+    of a device batch, computed on the GPU with plain torch FP64 (cuBLAS batched matmul,
+    grouped by (n, ldda)) — independent of libvbatched (the all-matrix check
+    of C5). A is regenerated by vbgen's device generator (F1, db's seed / gidx / non-SPD rule)
+    into scratch; L is the lower triangle of db's arena. Entries for info != 0 or n == 0 are NaN.
+    The FP64 rounding of L L^T adds O(1/sqrt(n)) to the ratio (validated against the
+    long-double oracle on a sample by the tests)."""
+    info = db.info()
+    out = np.full(db.B, np.nan)
+    keys = {}
+    for i in np.nonzero((info == 0) & (db.n > 0))[0]:
+        keys.setdefault((int(db.n[i]), int(db.ldda[i])), []).append(int(i))
+    eps = 2.0 ** -53
+    for (n, ld), idx in keys.items():
+        per = max(1, chunk_elems // (n * n))
+        for c0 in range(0, len(idx), per):
+            ii = idx[c0: c0 + per]
+            c = len(ii)
+            # L: the stored lower triangle of each matrix ([col][row] views of the arena)
+            M = torch.stack([db.arena.narrow(0, int(db.off[i]), ld * n).view(n, ld)[:, :n]
+                             for i in ii]).to(torch.float64)
+            L = torch.tril(M.transpose(1, 2))
+            # A: regenerated (lower triangle written, column-major, ld = n) into scratch
+            scratch = torch.zeros(c * n * n, dtype=torch.float64, device=db.device)
+            ptrs = torch.tensor([scratch.data_ptr() + 8 * n * n * k for k in range(c)],
+                                dtype=torch.int64, device=db.device)
+            dn = torch.full((c,), n, dtype=torch.int32, device=db.device)
+            dg = torch.tensor([int(db.gidx[i]) for i in ii], dtype=torch.int32, device=db.device)
+            vbdev.fill_f1(db.seed, c, dn.data_ptr(), dn.data_ptr(), ptrs.data_ptr(), dg.data_ptr(),
+                          db.nonspd_mod, 0, torch.cuda.current_stream().cuda_stream)
+            Alow = torch.tril(scratch.view(c, n, n).transpose(1, 2))
+            A = Alow + torch.tril(Alow, -1).transpose(1, 2)
+            R = A - torch.bmm(L, L.transpose(1, 2))
+            num = torch.linalg.matrix_norm(R)
+            den = torch.linalg.matrix_norm(A)
+            out[ii] = (num / (n * den * eps)).cpu().numpy()
+    return out

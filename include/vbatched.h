@@ -16,7 +16,9 @@
  *  - All int arguments are 32-bit. Offsets inside the library are computed in 64 bits.
  *  - Asynchronous: work is enqueued on `stream` (0 = legacy default stream); no host
  *    synchronisation and no device->host copy happens unless the routine says so. Internal
- *    workspace (O(batchCount) ints) is stream-ordered (cudaMallocAsync/cudaFreeAsync).
+ *    workspace (O(batchCount) ints) is stream-ordered (cudaMallocFromPoolAsync/cudaFreeAsync
+ *    on a memory pool the library creates per device; the caller's default pool and its
+ *    attributes are not touched).
  *  - Return value: 0 = enqueued; -p = host-scalar argument number p (1-based) is invalid,
  *    nothing enqueued; > 0 = a cudaError_t from the launch.
  *  - batchCount == 0 returns 0 and enqueues nothing.
@@ -60,7 +62,12 @@ typedef struct CUstream_st* vb_stream_t; /* == cudaStream_t */
  *  batchCount number of matrices (>= 0)                                      (-6 if < 0)
  *  max_n      an upper bound on every n_i (host)                              (-7 if < 0)
  *  stream     CUDA stream.
- * The other (unreferenced) strict triangle and rows n_i..ldda_i-1 are never read nor written.
+ * The other (unreferenced) strict triangle and rows n_i..ldda_i-1 are never WRITTEN. They are
+ * not read either, with one exception: the 16-byte TMA bulk copies of the n_i > 128 path round
+ * each column segment up to 16 bytes, so with uplo 'L' up to one padding element per column
+ * (row n_i when n_i is odd; it lies inside ldda_i) may be read. Its value never reaches any
+ * stored result, so NaN/Inf padding is harmless; it must only be readable memory (it is, since
+ * ldda_i >= n_i + 1 whenever the copy reaches it).
  * Matrices must not overlap. Returns 0 / -p / cudaError_t as described above.
  */
 int vbatched_dpotrf(char uplo, const int* d_n, double* const* dA_array, const int* d_ldda,
@@ -194,9 +201,18 @@ const char* vbatched_version(void);
  * one persistent kernel per non-empty size range). For benchmarks' launch accounting. */
 int vbatched_dpotrf_kernel_launches(int max_n);
 
+/* Names of the factorisation kernels one vbatched_dpotrf call with this max_n launches after
+ * the scan (for benchmark logs / roofline labels). Static string, never NULL. */
+const char* vbatched_dpotrf_kernel_names(int max_n);
+
 /* Pinned host memory helpers (cudaHostAlloc / cudaFreeHost) for the _host entry point. */
 void* vbatched_host_alloc(size_t bytes);
 int vbatched_host_free(void* p);
+
+/* vbatched_dpotrf_host keeps a per-device staging ring (device buffers up to workspace_bytes,
+ * pinned mirrors, 3 streams) between calls. This frees the current device's ring; call it
+ * outside any vbatched_dpotrf_host call. Returns 0 or a cudaError_t. */
+int vbatched_release_host_staging(void);
 
 #ifdef __cplusplus
 }

@@ -19,7 +19,8 @@ __all__ = [
     "vbatched_dpotrf", "vbatched_dpotrf_nomax", "vbatched_dpotrf_host",
     "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
-    "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "lib", "LIB_PATH", "VBatchedError",
+    "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "vbatched_dpotrf_kernel_names",
+    "vbatched_release_host_staging", "factor_kernel_names", "lib", "LIB_PATH", "VBatchedError",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -65,6 +66,10 @@ def lib() -> ctypes.CDLL:
         L.vbatched_version.restype = ctypes.c_char_p
         L.vbatched_dpotrf_kernel_launches.argtypes = [_i]
         L.vbatched_dpotrf_kernel_launches.restype = _i
+        L.vbatched_dpotrf_kernel_names.argtypes = [_i]
+        L.vbatched_dpotrf_kernel_names.restype = ctypes.c_char_p
+        L.vbatched_release_host_staging.argtypes = []
+        L.vbatched_release_host_staging.restype = _i
         L.vbatched_host_alloc.argtypes = [ctypes.c_size_t]
         L.vbatched_host_alloc.restype = _vp
         L.vbatched_host_free.argtypes = [_vp]
@@ -216,6 +221,17 @@ def vbatched_partition_lpt(h_n, ngpu: int):
 
 def vbatched_dpotrf_kernel_launches(max_n: int) -> int:
     return int(lib().vbatched_dpotrf_kernel_launches(int(max_n)))
+
+
+def vbatched_dpotrf_kernel_names(max_n: int) -> str:
+    return lib().vbatched_dpotrf_kernel_names(int(max_n)).decode()
+
+
+factor_kernel_names = vbatched_dpotrf_kernel_names
+
+
+def vbatched_release_host_staging() -> None:
+    _check(lib().vbatched_release_host_staging(), "vbatched_release_host_staging")
 
 
 def vbatched_version() -> str:

@@ -5,6 +5,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 #include <numeric>
 #include <vector>
 
@@ -14,20 +15,39 @@
 
 namespace vb {
 
-static bool g_pool_configured = false;
+// Stream-ordered workspace comes from a library-owned memory pool per device (created once,
+// release threshold 256 MB so that steady-state calls do no OS round trip). The caller's
+// default pool and its attributes are never touched.
+static cudaMemPool_t g_pool[64] = {};
+static std::mutex g_pool_mu;
+
+static cudaError_t lib_pool(cudaMemPool_t* out) {
+  int dev;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lock(g_pool_mu);
+  if (!g_pool[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t p;
+    if ((e = cudaMemPoolCreate(&p, &props)) != cudaSuccess) return e;
+    uint64_t thr = 256ull << 20;
+    cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+    g_pool[dev] = p;
+  }
+  *out = g_pool[dev];
+  return cudaSuccess;
+}
 
 cudaError_t ws_alloc(void** p, size_t bytes, cudaStream_t stream) {
-  if (!g_pool_configured) {
-    // Keep freed workspace in the device's default pool (no OS round trip per call).
-    int dev;
-    cudaMemPool_t pool;
-    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-      uint64_t thr = 256ull << 20;
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-    g_pool_configured = true;
-  }
-  return cudaMallocAsync(p, bytes, stream);
+  cudaMemPool_t pool;
+  cudaError_t e = lib_pool(&pool);
+  if (e != cudaSuccess) return e;
+  return cudaMallocFromPoolAsync(p, bytes, pool, stream);
 }
 
 cudaError_t ws_free(void* p, cudaStream_t stream) { return cudaFreeAsync(p, stream); }
@@ -264,6 +284,8 @@ const char* vbatched_version(void) {
 }
 
 int vbatched_dpotrf_kernel_launches(int max_n) { return max_n > 0 ? potrf_num_launches(max_n) : 0; }
+
+const char* vbatched_dpotrf_kernel_names(int max_n) { return potrf_kernel_names(max_n); }
 
 void* vbatched_host_alloc(size_t bytes) {
   void* p = nullptr;

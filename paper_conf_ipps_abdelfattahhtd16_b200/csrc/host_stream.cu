@@ -116,6 +116,7 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
   cudaError_t e = cudaSuccess;
   int dev = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return (int)e;
+  if (dev < 0 || dev >= kMaxDevices) return (int)cudaErrorInvalidDevice;
   Slot* slots = g_stage[dev].slots;
   const int nslots = std::min<int>(kBufs, (int)chunks.size());
   size_t need = 0;
@@ -202,4 +203,27 @@ extern "C" int vbatched_dpotrf_host(char uplo, const int* h_n, double* const* hA
     if (slots[s].stream) cudaStreamSynchronize(slots[s].stream);
   if (start_ev) cudaEventDestroy(start_ev);
   return (int)e;
+}
+
+// Frees the staging ring of the current device (device buffers, pinned mirrors, streams,
+// events) that vbatched_dpotrf_host keeps between calls. Safe to call at any time outside a
+// vbatched_dpotrf_host call; the next call re-creates what it needs.
+extern "C" int vbatched_release_host_staging(void) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return (int)e;
+  if (dev < 0 || dev >= kMaxDevices) return (int)cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lock(g_stage_mutex);
+  for (Slot& sl : g_stage[dev].slots) {
+    if (sl.stream) cudaStreamSynchronize(sl.stream);
+    if (sl.dbuf) cudaFree(sl.dbuf);
+    if (sl.dmeta) cudaFree(sl.dmeta);
+    if (sl.dptr) cudaFree(sl.dptr);
+    if (sl.hmeta) cudaFreeHost(sl.hmeta);
+    if (sl.hptr) cudaFreeHost(sl.hptr);
+    if (sl.done) cudaEventDestroy(sl.done);
+    if (sl.stream) cudaStreamDestroy(sl.stream);
+    sl = Slot();
+  }
+  return (int)cudaGetLastError();
 }

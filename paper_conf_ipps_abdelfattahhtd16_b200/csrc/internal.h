@@ -24,6 +24,7 @@ cudaError_t launch_potrf_paths(const int* d_n, float* const* dA, const int* d_ld
                                bool up, cudaStream_t stream);
 
 int potrf_num_launches(int max_n_hint);
+const char* potrf_kernel_names(int max_n_hint);  // the factorisation kernels after the scan
 // max_n <= 32: one warp kernel that validates and factors directly (no scan).
 cudaError_t launch_potrf_direct(const int* d_n, double* const* dA, const int* d_ldda, int* d_info,
                                 int batch, int max_n, bool up, cudaStream_t stream);

@@ -22,18 +22,21 @@
 //                        inverses from registers — the trtri + gemm TRSM of PAPER.md:760-772.
 //    Every element of L is written once; earlier columns are re-read once per panel (HBM
 //    re-read traffic ~ 8 n^3 / (6 NB) bytes per matrix).
-//  * potrf_small_kernel, 32 < n <= ts: one 2-warp CTA per matrix, 8 CTAs per SM, NB = 32,
-//    panel-update fragments straight from L2 (potrf_wsmall_kernel, one warp per matrix, is the
-//    VB_SMALL=1 alternative).
+//  * potrf_small_kernel, 32 < n <= ts: one (diagonal warp, off-diagonal warp) pair per matrix,
+//    two pairs per 4-warp CTA, 4 CTAs per SM, NB = 32 left-looking with look-ahead,
+//    panel-update fragments straight from L2.
 //  * potrf_warp_kernel, n <= 32: one warp per matrix, whole matrix in registers
 //    (the fused on-chip POTF2 of PAPER.md:551-560; one HBM read, one HBM write).
 // The kernels are chained with programmatic dependent launch: each releases its dependent
 // grid as soon as it starts, so the next range's CTAs take the SMs the previous kernel's
-// CTAs free at its tail (the smaller matrices come later in LPT order anyway).
+// CTAs free at its tail (the smaller matrices come later in LPT order anyway); every chained
+// grid waits (griddepcontrol.wait) for its upstream grid before it exits, so completion is
+// transitive and stream order holds for whatever the caller enqueues next.
 // Failed matrices (pivot <= 0 or NaN) stop at the failing column and report the LAPACK info
 // (SURVEY.md §8(c) readings #2-#3); nothing of them is touched again (a7).
 #include <algorithm>
 #include <cstdlib>
+#include <atomic>
 #include <mutex>
 
 #include "common.cuh"
@@ -789,6 +792,10 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
     }
     TL_END(tid == 0, t_tl, m, 30)
   }
+  // Chained without waiting (wait_upstream == 0): hold this grid's completion until the
+  // upstream grid has completed, so that completion stays transitive along the PDL chain and
+  // stream successors (workspace free, caller kernels) see every earlier grid finished.
+  if (!wait_upstream && threadIdx.x == 0) pdl_wait();
 }
 
 // =======================================================================================
@@ -799,7 +806,6 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
 // from L2 (__ldcg) into DMMA registers; the owning warp factors the diagonal block (POTF2 +
 // TRTRI in shared memory) and releases it to the other warp with a named barrier; TRSM runs
 // from registers and stores directly. One __syncthreads per panel.
-constexpr int kSmallWarps = 2;
 struct SmallSmem {
   double T[32][36];    // diagonal block, T[c][r]
   double inv[32][36];  // inv(L11) as TRSM B operand: inv[k][n] = X[n][k]
@@ -901,205 +907,6 @@ VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], E* __restr
       }
 }
 
-template <bool UP>
-__global__ void __launch_bounds__(32 * kSmallWarps, 8)
-    potrf_small_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
-                       const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                       const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
-                       int wait_upstream) {
-  __shared__ SmallSmem s;
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  if (wait_upstream) pdl_wait();
-  pdl_launch_dependents();
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (;;) {
-    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
-    __syncthreads();
-    const int it = s.item;
-    __syncthreads();
-    if (it >= count) break;
-    const int m = order[start + it];
-    const int n = d_n[m], ld = d_ldda[m];
-    double* A = dA[m];
-    VB_T0(t_m)
-    TL_BEGIN(t_tl)
-    for (int j0 = 0; j0 < n; j0 += 32) {
-      const int nb = min(32, n - j0);
-      const int nblk = (n - j0 + 31) / 32;
-      bool failed = false;
-      for (int b = warp; b < nblk; b += kSmallWarps) {
-        const int r0 = j0 + 32 * b;
-        double acc[4][4][2];
-        VB_T0(t_g)
-        small_panel_update<UP>(acc, A, n, ld, r0, j0, nb, b == 0, lane);
-        VB_ADD(0, t_g)
-        if (b == 0) {  // warp 0: the diagonal block
-          const int g = lane >> 2, q = lane & 3;
-#pragma unroll
-          for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-            for (int nt = 0; nt < 4; ++nt) {
-              s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
-              s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
-            }
-          __syncwarp();
-          VB_T0(t_p)
-          const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
-                                         s.wbuf, s.sv, s.tv);
-          VB_ADD(1, t_p)
-          VB_T0(t_i)
-          if (!info && nblk > 1)
-            trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
-          VB_ADD(2, t_i)
-          if (lane == 0) s.info = info;
-          failed = info != 0;
-          if (nblk > 1) bar_group_arrive(1, 32 * kSmallWarps);  // inv(L11) is ready
-        } else {
-          if (b == 1) {  // this warp's first block of the panel: wait for inv(L11)
-            bar_group(1, 32 * kSmallWarps);
-            failed = s.info != 0;
-          }
-          VB_T0(t_s)
-          if (!failed) small_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
-          VB_ADD(3, t_s)
-        }
-        if (failed) break;
-      }
-      VB_T0(t_b)
-      __syncthreads();  // the panel's L is stored (CTA scope) before the next panel reads it
-      VB_ADD(5, t_b)
-      if (s.info) {
-        if (tid == 0) d_info[m] = j0 + s.info;
-        break;
-      }
-    }
-    VB_ADD(4, t_m)
-    __syncthreads();
-    TL_END(tid == 0, t_tl, m, 20)
-  }
-}
-
-// Look-ahead small-matrix kernel (32 < n <= ts, the default): the same 2-warp CTA and NB = 32
-// blocks as potrf_small_kernel, but the warps are specialised. Warp 0 owns the diagonal
-// blocks only (panel update of the diagonal block, POTF2, TRTRI); warp 1 owns every block
-// below the diagonal (panel update + TRSM + store). Warp 0 starts panel p+1 as soon as warp 1
-// has stored block 1 of panel p (the rows of the next diagonal block), so the pivot chain of
-// panel p+1 overlaps warp 1's remaining blocks of panel p. Named barriers (64 threads):
-//   1 inv_ready(p)  warp 0 arrives after TRTRI(p) (or on failure), warp 1 syncs before TRSM;
-//   2 block1(p)     warp 1 arrives after storing block 1 of panel p, warp 0 syncs before the
-//                   diagonal update of panel p+1;
-//   3 inv_free(p)   warp 1 arrives after its last TRSM of panel p, warp 0 syncs before it
-//                   overwrites s.inv with inv(L11) of panel p+1 (single inverse buffer).
-// Arrivals and syncs are paired under the same conditions (panel p has blocks below it and
-// did not fail), so no barrier phase is left open across matrices.
-// One matrix by a (diagonal warp, off-diagonal warp) pair; named barriers bar0 (ready),
-// bar0+1 (block 1 stored), bar0+2 (inverse free).
-template <bool UP, typename E>
-VB_DEVINL void la_matrix(SmallSmem& s, int role, int lane, E* __restrict__ A, int n, int ld,
-                         int* info_out, int bar0) {
-  const int g = lane >> 2, q = lane & 3;
-  const int npan = (n + 31) / 32;
-  if (role == 0) {
-    bool pending_free = false;  // the other warp will arrive inv_free for the previous panel
-    for (int p = 0; p < npan; ++p) {
-      const int j0 = 32 * p, nb = min(32, n - j0);
-      const bool below = p + 1 < npan;
-      double acc[4][4][2];
-      VB_T0(t0)
-      small_acc_init<UP, E>(acc, A, n, ld, j0, j0, nb, true, lane);
-      if (p > 0) {
-        // columns of the panels before p-1 are final: their update runs while the other warp
-        // is still on block 1 of panel p-1; the newest 32 columns after block 1 is stored
-        small_kloop<UP, E>(acc, A, n, ld, j0, j0, 0, j0 - 32, lane);
-        VB_ADDW(0, t0)
-        VB_T0(t1)
-        bar_group(bar0 + 1, 64);  // block 1 of panel p-1 (= these rows) is stored
-        VB_ADDW(1, t1)
-        VB_T0(t2)
-        // the newest 32 columns: block 1 of panel p-1, which the other warp also left in s.T
-        // ([col][row], the stored values): a SYRK from shared memory instead of L2, same k order
-#pragma unroll
-        for (int ks = 0; ks < 8; ++ks) {
-          double fa[4], fb[4];
-#pragma unroll
-          for (int t = 0; t < 4; ++t) {
-            fb[t] = s.T[ks * 4 + q][t * 8 + g];
-            fa[t] = -fb[t];
-          }
-#pragma unroll
-          for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-            for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], fa[mt], fb[nt]);
-        }
-        __syncwarp();  // all reads of s.T done before it is overwritten with the tile
-        VB_ADDW(2, t2)
-      }
-#pragma unroll
-      for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-          s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
-          s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
-        }
-      __syncwarp();
-      VB_T0(t3)
-      const int info = potf2_block32<UP>(&s.T[0][0], 36, nb, lane, A + (size_t)j0 * ld + j0, ld,
-                                         s.wbuf, s.sv, s.tv);
-      VB_ADDW(3, t3)
-      VB_T0(t4)
-      if (pending_free) {  // the other warp is done with inv(L11) of panel p-1
-        bar_group(bar0 + 2, 64);
-        pending_free = false;
-      }
-      if (info) {
-        if (lane == 0) {
-          s.info = info;
-          *info_out = j0 + info;
-        }
-        if (below) bar_group_arrive(bar0, 64);  // the other warp reads s.info and stops
-        break;
-      }
-      if (!below) break;
-      trtri32_dmma_warp(&s.T[0][0], 36, s.tv, &s.inv[0][0], 36, s.S, LDS_T, lane);
-      if (lane == 0) s.info = 0;
-      bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready
-      VB_ADDW(4, t4)
-      pending_free = true;
-    }
-  } else {
-    for (int p = 0; p + 1 < npan; ++p) {  // panels with blocks below the diagonal
-      const int j0 = 32 * p;
-      const int nblk = (n - j0 + 31) / 32;
-      double acc[4][4][2];
-      VB_T0(t5)
-      small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
-      VB_ADDW(5, t5)
-      VB_T0(t6)
-      bar_group(bar0, 64);  // inv(L11) of panel p (or the failure)
-      VB_ADDW(6, t6)
-      if (s.info) break;
-      VB_T0(t7)
-      // block 1 = the rows of the next diagonal block: also leave it in s.T (free since the
-      // diagonal warp finished TRTRI(p); it reads it after the block1 barrier)
-      small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32, j0, lane, s.T);
-      __syncwarp();
-      VB_ADDW(7, t7)
-      bar_group_arrive(bar0 + 1, 64);  // block 1 stored: the diagonal warp may start panel p+1
-      for (int b = 2; b < nblk; ++b) {
-        VB_T0(t8)
-        small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
-        VB_ADDW(5, t8)
-        VB_T0(t9)
-        small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
-        VB_ADDW(7, t9)
-      }
-      bar_group_arrive(bar0 + 2, 64);  // done with s.inv of panel p
-    }
-  }
-}
-
 // Variant with the roles split by instruction mix (VB_SMALL=5): the diagonal warp runs only the
 // pivot chain (POTF2 + TRTRI of the tile in s.T); the off-diagonal warp does every DMMA update,
 // including the next diagonal tile: right after the TRSM of block 1 of panel p (the rows of the
@@ -1198,42 +1005,14 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
   }
 }
 
-template <bool UP, typename E = double>
-__global__ void __launch_bounds__(32 * kSmallWarps, 8)
-    potrf_small_la_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
-                          const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                          const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
-                          int range, int wait_upstream) {
-  __shared__ SmallSmem s;
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  if (wait_upstream) pdl_wait();
-  pdl_launch_dependents();
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (;;) {
-    if (tid == 0) s.item = atomicAdd(&ctrl->head[range], 1);
-    __syncthreads();
-    const int it = s.item;
-    __syncthreads();
-    if (it >= count) break;
-    const int m = order[start + it];
-    TL_BEGIN(t_tl)
-    la_matrix<UP, E>(s, warp, lane, dA[m], d_n[m], d_ldda[m], d_info + m, 1);
-    __syncthreads();
-    if (tid == 0) s.info = 0;
-    TL_END(tid == 0, t_tl, m, 21)
-  }
-}
-
 // The same pairs packed two per 4-warp CTA with the roles on fixed sub-partitions: warps 0/1 are
 // the diagonal warps of pair 0/1, warps 2/3 their off-diagonal warps (warp w runs on SMSP
 // w % 4), so the pivot chains share their sub-partitions only with other pivot chains, not
 // with the off-diagonal DMMA streams (tools/contention_bench.cu: a DMMA stream starves the
 // FP64 chain on its sub-partition). Each pair fetches its own matrices.
-template <bool UP, typename E = double, bool SPLIT = false>
+template <bool UP, typename E = double>
 __global__ void __launch_bounds__(128, 4)
-    potrf_small_la2_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
+    potrf_small_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                            const int* __restrict__ d_ldda, int* __restrict__ d_info,
                            const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
                            int range, int wait_upstream) {
@@ -1255,157 +1034,12 @@ __global__ void __launch_bounds__(128, 4)
     if (it >= count) break;
     const int m = order[start + it];
     TL_BEGIN(t_tl)
-    if constexpr (SPLIT)
-      la_matrix_v2<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
-    else
-      la_matrix<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
+    la_matrix_v2<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
     bar_group(tsync, 64);
     if (role == 0 && lane == 0) s.info = 0;
     TL_END(role == 0 && lane == 0, t_tl, m, 22)
   }
-}
-
-// =======================================================================================
-// Warp-per-matrix kernel for 32 < n <= ts (replaces the 2-warp small kernel by default):
-// one warp factors one matrix alone — no inter-warp synchronisation — and 16 single-warp
-// CTAs share an SM (~12 KB of shared memory each), so 16 small matrices are in flight per
-// SM. NB = 32 left-looking; 32-row blocks in sequence; panel-update fragments straight from
-// L2; POTF2 of the diagonal block in registers; the TRSM is a block substitution on DMMA
-// with the four 8x8 diagonal-block inverses of L11 (no full 32x32 inverse buffer):
-//   X_b = (C_b - sum_{c<b} X_c L_bc^T) inv(L_bb)^T,  b = 0..3 (8-column blocks).
-constexpr int LDW = 36;
-struct WSmem {
-  double T[32][LDW];       // diagonal block; L11 after POTF2
-  double inv8[4][8][9];    // inv(L_bb) as B operand: inv8[b][k][n] = inv(L_bb)[n][k]
-  double wbuf[64];
-  double sv[32];
-  double tv[32];
-};
-
-// Inverses of the four 8x8 diagonal blocks of L11 (T, tv = 1/l_cc): lane = (b, c) computes
-// column c of inv(L_bb) by substitution.
-VB_DEVINL void inv8_blocks(WSmem& s, int lane) {
-  const int b = lane >> 3, c = lane & 7, o = 8 * b;
-  double x[8];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    double acc = 0.0;
-#pragma unroll
-    for (int k = 0; k < i; ++k) acc = fma(s.T[o + k][o + i], x[k], acc);
-    const double r = s.tv[o + i];
-    x[i] = (i < c) ? 0.0 : ((i == c) ? r : -acc * r);
-  }
-#pragma unroll
-  for (int i = 0; i < 8; ++i) s.inv8[b][c][i] = x[i];  // [k=c][n=i] = inv[i][c]
-  __syncwarp();
-}
-
-// In-register TRSM of a 32 x 32 C block (C-fragment layout) against L11 by 8-column block
-// substitution; result stored to global rows < n.
-template <bool UP>
-VB_DEVINL void wsmall_trsm_store(WSmem& s, double (&acc)[4][4][2], double* __restrict__ A, int n,
-                                 int ld, int r0, int j0, int lane) {
-  const int g = lane >> 2, q = lane & 3;
-#pragma unroll
-  for (int b = 0; b < 4; ++b) {
-    // C_b -= X_c L_bc^T for c < b:  B[k][n] = L[8b+n][8c+k] = T[8c+k][8b+n]
-#pragma unroll
-    for (int c = 0; c < b; ++c) {
-#pragma unroll
-      for (int ks = 0; ks < 2; ++ks) {
-        const double fb = s.T[8 * c + 4 * ks + q][8 * b + g];
-#pragma unroll
-        for (int mt = 0; mt < 4; ++mt) {
-          const double fa = -cfrag_to_afrag(acc[mt][c][0], acc[mt][c][1], ks, lane);
-          dmma(acc[mt][b], fa, fb);
-        }
-      }
-    }
-    // X_b = C_b inv(L_bb)^T
-    double x[4][2];
-#pragma unroll
-    for (int mt = 0; mt < 4; ++mt) x[mt][0] = x[mt][1] = 0.0;
-#pragma unroll
-    for (int ks = 0; ks < 2; ++ks) {
-      const double fb = s.inv8[b][4 * ks + q][g];
-#pragma unroll
-      for (int mt = 0; mt < 4; ++mt) {
-        const double fa = cfrag_to_afrag(acc[mt][b][0], acc[mt][b][1], ks, lane);
-        dmma(x[mt], fa, fb);
-      }
-    }
-#pragma unroll
-    for (int mt = 0; mt < 4; ++mt) {
-      acc[mt][b][0] = x[mt][0];
-      acc[mt][b][1] = x[mt][1];
-    }
-  }
-#pragma unroll
-  for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-    for (int nt = 0; nt < 4; ++nt)
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int row = r0 + mt * 8 + g, col = nt * 8 + 2 * q + h;
-        if (row < n) A[gix<UP>(row, j0 + col, ld)] = acc[mt][nt][h];
-      }
-}
-
-template <bool UP>
-__global__ void __launch_bounds__(32, 16)
-    potrf_wsmall_kernel(const int* __restrict__ d_n, double* const* __restrict__ dA,
-                        const int* __restrict__ d_ldda, int* __restrict__ d_info,
-                        const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order, int range,
-                        int wait_upstream) {
-  __shared__ __align__(16) WSmem s;
-  Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
-  if (wait_upstream) pdl_wait();
-  pdl_launch_dependents();
-  const int count = *(volatile const int*)&ctrl->count[range];
-  const int start = *(volatile const int*)&ctrl->start[range];
-  const int lane = threadIdx.x;
-  for (;;) {
-    int it = 0;
-    if (lane == 0) it = atomicAdd(&ctrl->head[range], 1);
-    it = __shfl_sync(kFull, it, 0);
-    if (it >= count) break;
-    const int m = order[start + it];
-    const int n = d_n[m], ld = d_ldda[m];
-    double* A = dA[m];
-    for (int j0 = 0; j0 < n; j0 += 32) {
-      const int nb = min(32, n - j0);
-      const int nblk = (n - j0 + 31) / 32;
-      int info = 0;
-      for (int b = 0; b < nblk; ++b) {
-        const int r0 = j0 + 32 * b;
-        double acc[4][4][2];
-        small_panel_update<UP>(acc, A, n, ld, r0, j0, nb, b == 0, lane);
-        if (b == 0) {
-          const int g = lane >> 2, q = lane & 3;
-#pragma unroll
-          for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-            for (int nt = 0; nt < 4; ++nt) {
-              s.T[nt * 8 + 2 * q][mt * 8 + g] = acc[mt][nt][0];
-              s.T[nt * 8 + 2 * q + 1][mt * 8 + g] = acc[mt][nt][1];
-            }
-          __syncwarp();
-          info = potf2_block32<UP>(&s.T[0][0], LDW, nb, lane, A + (size_t)j0 * ld + j0, ld, s.wbuf,
-                               s.sv, s.tv);
-          if (info) break;
-          if (nblk > 1) inv8_blocks(s, lane);
-        } else {
-          wsmall_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
-        }
-      }
-      if (info) {
-        if (lane == 0) d_info[m] = j0 + info;
-        break;
-      }
-      // this warp stored the whole panel: its own later __ldcg reads see it (same thread order)
-      __syncwarp();
-    }
-  }
+  if (!wait_upstream && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1465,6 +1099,7 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
       potrf_warp_matrix<32, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     TL_END(lane == 0, t_tl, m, 40)
   }
+  if (!wait_upstream && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
 }
 
 // Direct warp path for batches whose max_n <= 32 (no scan, no sort: with every matrix this
@@ -1496,26 +1131,29 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
 }
 
 // ---------------------------------------------------------------------------------------
-static int g_num_sms = 0;
-static int g_occ64 = 0;
-static int g_ts = -1;
-static int g_occ_small = 0, g_occ_wsmall = 0;
-static int g_small = -1;
+// Host-side state. The size threshold is read once per process (std::call_once); the kernel
+// attributes (dynamic shared memory limits) are set once per device (bit per ordinal, under a
+// mutex); occupancies and the SM count are those of the first device initialised (the pool's
+// GPUs are identical B200s) and are published through atomics.
+static std::atomic<int> g_num_sms{0};
+static std::atomic<int> g_occ64{0}, g_occ64s{0};
+static int g_ts = 128;
+static std::once_flag g_ts_once;
 
 // Size threshold: n > ts takes the blocked NB=64 kernel, 32 < n <= ts the small-matrix kernel
 // (env VB_TS; default 128, measured: the blocked kernel beats the small kernel above 128 and
 // loses below, tools/cfgtime.py sweeps in profiles/r01).
 int potrf_ts() {
-  if (g_ts < 0) {
+  std::call_once(g_ts_once, [] {
     const char* e = getenv("VB_TS");
-    g_ts = e ? atoi(e) : 128;
-    if (g_ts < kWarpMaxN) g_ts = kWarpMaxN;
-  }
+    int t = e ? atoi(e) : 128;
+    g_ts = t < kWarpMaxN ? kWarpMaxN : t;
+  });
   return g_ts;
 }
 
 template <class C>
-static cudaError_t setup_blocked(int* occ) {
+static cudaError_t setup_blocked(std::atomic<int>* occ_out) {
   cudaError_t e = cudaFuncSetAttribute(potrf_blocked3_kernel<C, false>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)sizeof(Smem2<C>));
@@ -1523,17 +1161,13 @@ static cudaError_t setup_blocked(int* occ) {
   e = cudaFuncSetAttribute(potrf_blocked3_kernel<C, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Smem2<C>));
   if (e != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, potrf_blocked3_kernel<C, false>,
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, potrf_blocked3_kernel<C, false>,
                                                     32 * (C::WARPS + 1), sizeof(Smem2<C>));
-  if (*occ < 1) *occ = 1;
+  occ_out->store(occ < 1 ? 1 : occ);
   return e;
 }
 
-static int g_occ64s = 0;
-
-// Kernel attributes (dynamic shared memory limits) are per device: the setup runs once for every
-// device the library is called on (bit per ordinal); occupancies and the SM count are those of
-// the first device (the pool's GPUs are identical B200s).
 static unsigned long long g_dev_ready = 0;
 static std::mutex g_init_mu;
 
@@ -1541,29 +1175,17 @@ static cudaError_t init_device_info() {
   int dev;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  const unsigned long long bit = dev < 64 ? 1ull << dev : 0ull;
-  if (g_num_sms && (g_dev_ready & bit)) return cudaSuccess;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  const unsigned long long bit = 1ull << dev;
   std::lock_guard<std::mutex> lock(g_init_mu);
-  if (g_num_sms && (g_dev_ready & bit)) return cudaSuccess;
+  if (g_dev_ready & bit) return cudaSuccess;
   int sms = 0;
   e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
   if ((e = setup_blocked<Cfg64d>(&g_occ64)) != cudaSuccess) return e;
   if ((e = setup_blocked<Cfg64s>(&g_occ64s)) != cudaSuccess) return e;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_small, potrf_small_la_kernel<false>,
-                                                    32 * kSmallWarps, 0);
-  if (e != cudaSuccess) return e;
-  if (g_occ_small < 1) g_occ_small = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_occ_wsmall, potrf_wsmall_kernel<false>, 32,
-                                                    0);
-  if (e != cudaSuccess) return e;
-  if (g_occ_wsmall < 1) g_occ_wsmall = 1;
-  {
-    const char* v = getenv("VB_SMALL");
-    g_small = v ? atoi(v) : 5;
-  }
   potrf_ts();
-  g_num_sms = sms;
+  g_num_sms.store(sms);
   g_dev_ready |= bit;
   return cudaSuccess;
 }
@@ -1598,58 +1220,29 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
   cfg.numAttrs = 1;
   cfg.stream = stream;
   int wait = 1;  // the first factorisation kernel after the scan waits for it
-  if (max_n_hint > g_ts) {
-    const int occ = sizeof(E) == 8 ? g_occ64 : g_occ64s;
+  if (max_n_hint > potrf_ts()) {
+    const int occ = sizeof(E) == 8 ? g_occ64.load() : g_occ64s.load();
     cfg.blockDim = dim3(32 * (C::WARPS + 1));
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * occ)));
+    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms.load() * occ)));
     cfg.dynamicSmemBytes = sizeof(Smem2<C>);
     e = cudaLaunchKernelEx(&cfg, up ? potrf_blocked3_kernel<C, true> : potrf_blocked3_kernel<C, false>,
                            d_n, dA, d_ldda, d_info, ctrl, order, 0, wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
+  const int sms = g_num_sms.load();
   if (max_n_hint > kWarpMaxN) {
-    cfg.blockDim = dim3(32 * kSmallWarps);
-    cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_small)));
+    cfg.blockDim = dim3(128);
+    cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, sms * 4)));
     cfg.dynamicSmemBytes = 0;
-    if constexpr (sizeof(E) == 8) {
-      if (g_small == 5) {
-        cfg.blockDim = dim3(128);
-        cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
-        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, double, true>
-                                        : potrf_small_la2_kernel<false, double, true>,
-                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-      } else if (g_small == 4) {
-        cfg.blockDim = dim3(128);
-        cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
-        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true> : potrf_small_la2_kernel<false>,
-                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-      } else if (g_small == 3) {
-        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la_kernel<true> : potrf_small_la_kernel<false>,
-                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-      } else if (g_small == 2) {
-        e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true> : potrf_small_kernel<false>, d_n,
-                               dA, d_ldda, d_info, ctrl, order, 1, wait);
-      } else {
-        cfg.blockDim = dim3(32);
-        cfg.gridDim = dim3(std::max(1, std::min(batch, g_num_sms * g_occ_wsmall)));
-        e = cudaLaunchKernelEx(&cfg, up ? potrf_wsmall_kernel<true> : potrf_wsmall_kernel<false>,
-                               d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-      }
-    } else {
-      cfg.blockDim = dim3(128);
-      cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, g_num_sms * 4)));
-      e = cudaLaunchKernelEx(&cfg, up ? potrf_small_la2_kernel<true, E, true>
-                                      : potrf_small_la2_kernel<false, E, true>,
-                             d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
-    }
+    e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true, E> : potrf_small_kernel<false, E>,
+                           d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
     if (e != cudaSuccess) return e;
     wait = 0;
   }
   const int warps = std::max(1, batch);
   cfg.blockDim = dim3(32 * kWarpsPerCta);
-  cfg.gridDim = dim3(std::max(1, std::min((warps + kWarpsPerCta - 1) / kWarpsPerCta,
-                                          g_num_sms * 8)));
+  cfg.gridDim = dim3(std::max(1, std::min((warps + kWarpsPerCta - 1) / kWarpsPerCta, sms * 8)));
   cfg.dynamicSmemBytes = 0;
   return cudaLaunchKernelEx(&cfg, up ? potrf_warp_kernel<true, E> : potrf_warp_kernel<false, E>,
                             d_n, dA, d_ldda, d_info, ctrl, order, wait);
@@ -1668,10 +1261,10 @@ cudaError_t launch_potrf_paths(const int* d_n, float* const* dA, const int* d_ld
 
 void potrf_occupancy(int* out4) {
   init_device_info();
-  out4[0] = g_occ64;
+  out4[0] = g_occ64.load();
   out4[1] = Cfg64d::WARPS;
   out4[2] = 0;  // (no separate NB=32 range)
-  out4[3] = g_small >= 4 ? 4 : (g_small >= 2 ? g_occ_small : g_occ_wsmall);
+  out4[3] = 4;  // small kernel: 4 CTAs (8 matrices) per SM
 }
 
 int potrf_num_launches(int max_n_hint) {
@@ -1680,12 +1273,19 @@ int potrf_num_launches(int max_n_hint) {
   return 3 + (max_n_hint > potrf_ts() ? 1 : 0);
 }
 
+const char* potrf_kernel_names(int max_n_hint) {
+  if (max_n_hint <= 0) return "";
+  if (max_n_hint <= kWarpMaxN) return "potrf_warp_direct_kernel";
+  if (max_n_hint <= potrf_ts()) return "potrf_small_kernel + potrf_warp_kernel";
+  return "potrf_blocked3_kernel + potrf_small_kernel + potrf_warp_kernel";
+}
+
 template <typename E>
 static cudaError_t launch_direct(const int* d_n, E* const* dA, const int* d_ldda, int* d_info,
                                  int batch, int max_n, bool up, cudaStream_t stream) {
   cudaError_t e = init_device_info();
   if (e != cudaSuccess) return e;
-  const int grid = std::max(1, std::min((batch + kWarpsPerCta - 1) / kWarpsPerCta, g_num_sms * 16));
+  const int grid = std::max(1, std::min((batch + kWarpsPerCta - 1) / kWarpsPerCta, g_num_sms.load() * 16));
   if (up)
     potrf_warp_direct_kernel<true, E><<<grid, 32 * kWarpsPerCta, 0, stream>>>(d_n, dA, d_ldda,
                                                                              d_info, batch, max_n);

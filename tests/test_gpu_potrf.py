@@ -150,11 +150,9 @@ print("OK")
     assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
 
 
-@pytest.mark.parametrize("small", ["1", "2", "3", "4", "5"])
-def test_small_kernel_variants(small):
-    """Both small-matrix kernels (VB_SMALL=1 warp-per-matrix, 2 = two warps per matrix) on C2
-    sizes plus failing pivots in every 8-column sub-block (subprocess: the variant is read at
-    first use)."""
+def test_small_kernel_c2_sizes_and_failures():
+    """The small-matrix kernel (32 < n <= 128) on C2 sizes plus failing pivots in every 8-column
+    sub-block (subprocess, so that a hang in the look-ahead barriers cannot wedge the run)."""
     import subprocess
     import sys
     code = f"""
@@ -181,9 +179,7 @@ for i in range(len(n)):
     assert r["ok"], (i, r)
 print("OK")
 """
-    env = dict(os.environ, VB_SMALL=small)
-    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env,
-                         timeout=600)
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600)
     assert out.returncode == 0 and "OK" in out.stdout, out.stdout[-2000:] + out.stderr[-3000:]
 
 
@@ -249,7 +245,9 @@ def test_config_full_parity(cfg):
 
 def test_c5_full_size_sampled():
     """C5 at BASELINE size (40000 x U{1..1024}, 112 GB) in the bench launch configuration;
-    every info must be 0; a deterministic sample is compared with the oracle."""
+    every info must be 0; a deterministic sample is compared with the oracle element by
+    element, and EVERY matrix's backward error is checked (<= 10, north_star) by the
+    independent torch FP64 checker (harness.gpu_backward_errors)."""
     free, _ = torch.cuda.mem_get_info()
     c = vbgen.CONFIGS["C5"]
     n = vbgen.sizes(c)
@@ -263,6 +261,12 @@ def test_c5_full_size_sampled():
     order = np.argsort(-n, kind="stable")
     sample = list(order[:4]) + list(range(0, db.B, 4001)) + list(order[-3:])
     _check_batch(db, idxs=sample)
+    from harness import gpu_backward_errors
+    be = gpu_backward_errors(db)
+    assert np.all(np.isfinite(be)), int(np.sum(~np.isfinite(be)))
+    print(f"C5 all-matrix backward error: max {be.max():.3f}, mean {be.mean():.4f}, "
+          f"p99 {np.percentile(be, 99):.3f} over {db.B} matrices")
+    assert be.max() <= 10.0, (int(np.argmax(be)), float(be.max()))
     del db
     torch.cuda.empty_cache()
 

@@ -442,3 +442,118 @@ def test_spotrf_oracle_vs_fp64_and_lapack():
     A = vbgen.f1_matrix(13, 7, 90).astype(np.float32)
     A[40, 40] = -A[40, 40]
     assert oracle.spotrf(A)[1] == 41
+
+
+# ---------------------------------------------------------------- the parity gates themselves
+# The two gate functions every GPU parity test relies on are pinned here against closed forms
+# computed independently (exact rationals / hand arithmetic), so that a gate that returned 0,
+# used eps = 2^-52 instead of 2^-53, dropped the factor n, or read the wrong triangle would fail.
+def _bwd_closed_form(A, Lg, nb, eps):
+    """||A - Lg Lg^T||_F / (nb ||A||_F eps) on the leading nb block, exact rational sums
+    (Fractions) and one final float sqrt: independent of the oracle's long-double loop."""
+    Af = [[Fraction(float(A[max(i, j), min(i, j)])) for j in range(nb)] for i in range(nb)]
+    Lf = [[Fraction(float(Lg[i, k])) if k <= i else Fraction(0) for k in range(nb)]
+          for i in range(nb)]
+    num = Fraction(0)
+    den = Fraction(0)
+    for i in range(nb):
+        for j in range(nb):
+            s = sum((Lf[i][k] * Lf[j][k] for k in range(nb)), Fraction(0))
+            d = Af[i][j] - s
+            num += d * d
+            den += Af[i][j] * Af[i][j]
+    return math.sqrt(num) / (nb * math.sqrt(den) * eps)
+
+
+def _int_spd(n, seed):
+    rng = np.random.default_rng(seed)
+    L = np.tril(rng.integers(-3, 4, size=(n, n)), -1).astype(np.float64)
+    L[np.arange(n), np.arange(n)] = rng.integers(1, 5, size=n)
+    return L, np.asfortranarray(L @ L.T)  # exact small integers
+
+
+def test_backward_error_gate_closed_form():
+    """oracle_backward_error on an exact A = L L^T with a known perturbation of L: equals the
+    closed form ||A - Lg Lg^T||_F / (n ||A||_F 2^-53) to 1e-9 relative (SURVEY §8(c) #13)."""
+    L, A = _int_spd(7, 41)
+    assert oracle.backward_error(A, np.asfortranarray(L), 0) == 0.0  # exact factor -> 0
+    for (p, q, d) in [(3, 1, 2.0 ** -40), (6, 6, -(2.0 ** -37)), (0, 0, 2.0 ** -45)]:
+        Lg = np.asfortranarray(L.copy())
+        Lg[p, q] += d
+        got = oracle.backward_error(A, Lg, 0)
+        exp = _bwd_closed_form(A, Lg, 7, 2.0 ** -53)
+        assert got == pytest.approx(exp, rel=1e-9), (p, q, got, exp)
+        # the same number by hand for a single perturbed entry: Delta = d (l_q e_p^T + e_p l_q^T)
+        # + d^2 e_p e_p^T with l_q = column q of L (row p's own entry included)
+        lq = L[:, q].copy()
+        D = d * (np.outer(lq, np.eye(7)[p]) + np.outer(np.eye(7)[p], lq))
+        D[p, p] += d * d
+        hand = np.sqrt(np.sum(D * D)) / (7 * np.sqrt(np.sum(A * A)) * 2.0 ** -53)
+        assert got == pytest.approx(hand, rel=1e-6)
+    # eps = 2^-52 or a dropped n would be off by exactly 2x / 7x
+    Lg = np.asfortranarray(L.copy())
+    Lg[4, 2] += 2.0 ** -40
+    got = oracle.backward_error(A, Lg, 0)
+    assert got != pytest.approx(_bwd_closed_form(A, Lg, 7, 2.0 ** -52), rel=0.1)
+    assert got != pytest.approx(_bwd_closed_form(A, Lg, 7, 2.0 ** -53) * 7, rel=0.1)
+
+
+def test_backward_error_gate_triangles_and_leading_block():
+    """Only A's lower triangle and Lg's lower triangle are read; on info > 0 only the leading
+    (info-1) block counts (SURVEY §8(c) readings #3, #13)."""
+    L, A = _int_spd(6, 43)
+    Ab = np.asfortranarray(A.copy())
+    Ab[np.triu_indices(6, 1)] = np.nan  # strict upper of A: never read
+    Lg = np.asfortranarray(L.copy())
+    Lg[np.triu_indices(6, 1)] = np.nan  # strict upper of the factor: taken as zero
+    Lg[2, 1] += 2.0 ** -40
+    got = oracle.backward_error(Ab, Lg, 0)
+    assert got == pytest.approx(_bwd_closed_form(A, Lg, 6, 2.0 ** -53), rel=1e-9)
+    # info = 4: the leading 3x3 block only; a perturbation in row 4 does not count
+    Lg2 = np.asfortranarray(L.copy())
+    Lg2[4, 1] += 1.0
+    assert oracle.backward_error(A, Lg2, 4) == 0.0
+    Lg2[1, 0] += 2.0 ** -40
+    assert oracle.backward_error(A, Lg2, 4) == pytest.approx(
+        _bwd_closed_form(A, Lg2, 3, 2.0 ** -53), rel=1e-9)
+
+
+def test_backward_error_f32_gate_closed_form():
+    """backward_error_f32 is the same ratio with eps32 = 2^-24."""
+    L, A = _int_spd(5, 47)
+    Lg = np.asfortranarray(L.copy())
+    Lg[3, 2] += 2.0 ** -20
+    assert oracle.backward_error_f32(A, Lg, 0) == pytest.approx(
+        _bwd_closed_form(A, Lg, 5, 2.0 ** -24), rel=1e-9)
+
+
+def test_rowscaled_gate_closed_form():
+    """rowscaled_diff = max_{i>=j} |Lg_ij - Lo_ij| / ||Lo(i, 0:i)||_2 on the leading nb block
+    (SURVEY §8(c) reading #14), on hand-built rows with norms 3, 5, 3, 13."""
+    Lo = np.array([[3.0, 0, 0, 0],
+                   [3.0, 4.0, 0, 0],
+                   [1.0, 2.0, 2.0, 0],
+                   [3.0, 4.0, 12.0, 0.0]])  # row norms 3, 5, 3, 13
+    assert oracle.rowscaled_diff(Lo, Lo, 4) == 0.0
+    Lg = Lo.copy()
+    Lg[1, 0] += 1e-6       # 1e-6 / 5
+    assert oracle.rowscaled_diff(Lg, Lo, 4) == pytest.approx(2e-7, rel=1e-12)
+    Lg[2, 2] -= 3e-5       # 3e-5 / 3 = 1e-5 (the max)
+    assert oracle.rowscaled_diff(Lg, Lo, 4) == pytest.approx(1e-5, rel=1e-9)
+    Lg[3, 2] = -12.0       # sign flip: 24 / 13
+    assert oracle.rowscaled_diff(Lg, Lo, 4) == pytest.approx(24 / 13, rel=1e-12)
+    # the strict upper triangle and rows/cols beyond nb are not compared
+    Lh = Lo.copy()
+    Lh[0, 3] = 1e9
+    Lh[3, 3] = 7.0
+    assert oracle.rowscaled_diff(Lh, Lo, 3) == 0.0
+    assert oracle.rowscaled_diff(Lh, Lo, 4) == pytest.approx(7 / 13, rel=1e-12)
+    # a zero row of the oracle's factor scales by 1 (absolute difference)
+    Z = np.zeros((2, 2))
+    Zg = Z.copy()
+    Zg[1, 0] = 2.5e-3
+    assert oracle.rowscaled_diff(Zg, Z, 2) == pytest.approx(2.5e-3, rel=1e-12)
+    # a NaN in the compared part must fail the gate (compare_with_oracle uses <= 1e-10)
+    Ln = Lo.copy()
+    Ln[2, 1] = np.nan
+    assert not (oracle.rowscaled_diff(Ln, Lo, 4) <= 1e-10)

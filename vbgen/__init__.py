@@ -108,6 +108,22 @@ def f1_matrix(seed: int, gidx: int, n: int, nonspd: bool = False) -> np.ndarray:
     return np.asfortranarray(a)
 
 
+def f2_matrix(seed: int, gidx: int, n: int, kappa: float = 1e4) -> np.ndarray:
+    """Family F2 (SURVEY.md §8(c) reading #9, parity only): Q diag(lambda) Q^T with Q the
+    orthogonal factor of a seeded Gaussian matrix and lambda log-uniform in [1, kappa]
+    (endpoints included, so kappa(A) ~= kappa), symmetrised. Input generation only."""
+    if n == 0:
+        return np.zeros((0, 0), order="F")
+    rng = np.random.default_rng([seed, gidx, n, 0xF2])
+    Q, _ = np.linalg.qr(rng.standard_normal((n, n)))
+    lam = 10.0 ** rng.uniform(0.0, np.log10(kappa), n)
+    lam[0] = 1.0
+    if n > 1:
+        lam[-1] = kappa
+    A = (Q * lam) @ Q.T
+    return np.asfortranarray((A + A.T) / 2)
+
+
 def config_matrix(cfg: Config | str, gidx: int, n: int | None = None) -> np.ndarray:
     if isinstance(cfg, str):
         cfg = CONFIGS[cfg]
