@@ -1,0 +1,15 @@
+#!/bin/bash
+# compute-sanitizer memcheck / synccheck / initcheck / racecheck on the C1 and mixed cases
+# (tools/sanitize_case.py). Logs -> gpurun_out/san/ (copied to profiles/r02/ when judged).
+cd "$(dirname "$0")/.."
+O=gpurun_out/san; mkdir -p $O
+for tool in memcheck synccheck initcheck racecheck; do
+  for case in c1 mixed; do
+    extra=""
+    [ $tool = memcheck ] && extra=""
+    [ $tool = initcheck ] && extra="--track-unused-memory no"
+    timeout 900 compute-sanitizer --tool $tool $extra --kernel-name kns=_ZN2vb --error-exitcode 9 \
+      python tools/sanitize_case.py $case > $O/${tool}_${case}.log 2>&1
+    echo "$tool $case rc=$?" | tee -a $O/summary.txt
+  done
+done
