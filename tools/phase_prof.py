@@ -39,6 +39,16 @@ db.dpotrf()
 e1.record()
 torch.cuda.synchronize()
 L.vbatched_debug_phases(ctypes.addressof(out), 1)
+if os.environ.get("QUAD"):  # quad small kernel: slots 0-2 chain warp, 3-6 the 3 DMMA warps, 7 all 4
+    names = ["chain:wait_tile", "chain:potf2", "chain:trtri", "dmma:pre_kloop", "dmma:wait_inv",
+             "dmma:strips", "dmma:tile_build", "all:matrix"]
+    scale = [1, 1, 1, 1 / 3, 1 / 3, 1 / 3, 1 / 3, 1 / 4]
+    tot = out[7] / 4
+    print(f"{cfg} kernel {e0.elapsed_time(e1):.3f} ms; cycles per warp of each role (sum over CTAs)")
+    for i, nm in enumerate(names):
+        v = out[i] * scale[i]
+        print(f"  {nm:18s} {v:16.0f}  {100.0 * v / max(tot, 1):6.1f} % of matrix time")
+    sys.exit(0)
 names = (["gemm", "potf2", "trtri", "trsm", "matrix_total", "panel_bar"] if os.environ.get("SMALL") else
          ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "acc_init"])
 tot = out[4]

@@ -4,6 +4,7 @@
 // L2 loads, hog kind 1) until the chain warp is done. Prints the chain's cycles per case.
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o tools/pipe_share_bench tools/pipe_share_bench.cu
 #include "../paper_conf_ipps_abdelfattahhtd16_b200/csrc/potrf.cu"
+#include "quad_experiment.cuh"
 #include <cstdio>
 
 using namespace vb;
@@ -60,6 +61,14 @@ __global__ void share_kernel(double* out, const double* src, long long* cyc, int
       double s = 0;
       for (int i = 0; i < 16; ++i) s += acc[i][0] + acc[i][1];
       out[(size_t)gridDim.x * 1024 + 64 + threadIdx.x] = s;
+    } else if (hog_kind == 2) {  // the quad kernel's strip k-loop: L2 fragments + DMMA
+      double acc[2][4][2] = {};
+      const double* A = src + (((size_t)blockIdx.x * 8 + warp) * 4096) % ((1 << 20) - 4096);
+      while (!stop) strip_kloop_t<false, double, 2, 4, -1>(acc, A, 64, 64, 0, 16, 0, 48, lane);
+      double s = 0;
+      for (int i = 0; i < 2; ++i)
+        for (int j = 0; j < 4; ++j) s += acc[i][j][0] + acc[i][j][1];
+      out[(size_t)gridDim.x * 1024 + 64 + threadIdx.x] = s;
     } else {  // L2 load stream (LDG.64 __ldcg), 8 in flight per lane
       double s = 0;
       size_t off = ((size_t)blockIdx.x * 8 + warp) * 4096 + lane;
@@ -90,8 +99,8 @@ int main() {
                     {(1 << 1) | (1 << 2) | (1 << 3), "SMSP1+2+3"},
                     {(1 << 1) | (1 << 2) | (1 << 3) | (1 << 5) | (1 << 6) | (1 << 7), "SMSP1+2+3 x2"},
                     {0xFE, "all incl SMSP0"}};
-  for (int kind = 0; kind < 2; ++kind)
-    for (int mode = 0; mode < 4; ++mode)
+  for (int kind = 0; kind < 3; ++kind)
+    for (int mode = 0; mode < (kind == 2 ? 1 : 4); ++mode)
       for (const H& h : hogs) {
         share_kernel<<<148, 256>>>(out, src, cyc, h.mask, mode, kind, 8);
         if (cudaDeviceSynchronize() != cudaSuccess) { printf("launch failed\n"); return 1; }
@@ -100,7 +109,7 @@ int main() {
         double s = 0;
         for (int b = 0; b < 148; ++b) s += c[b];
         printf("{\"chain\":\"%s\",\"hog\":\"%s\",\"hog_warps\":\"%s\",\"cycles\":%.0f}\n", modes[mode],
-               kind ? "ldg_l2" : "dmma", h.what, s / 148);
+               kind == 2 ? "strip_kloop" : (kind ? "ldg_l2" : "dmma"), h.what, s / 148);
       }
   printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
   return 0;

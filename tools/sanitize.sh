@@ -5,9 +5,9 @@ cd "$(dirname "$0")/.."
 O=gpurun_out/san; mkdir -p $O
 for tool in memcheck synccheck initcheck racecheck; do
   for case in c1 mixed; do
-    extra=""
-    [ $tool = memcheck ] && extra=""
-    [ $tool = initcheck ] && extra="--track-unused-memory no"
+    # API-call error reports are off: torch's lazy module loading probes cuKernelGetFunction
+    # with handles of kernels it has not loaded (CUDA_ERROR_INVALID_HANDLE), unrelated to ours
+    extra="--report-api-errors no"
     timeout 900 compute-sanitizer --tool $tool $extra --kernel-name kns=_ZN2vb --error-exitcode 9 \
       python tools/sanitize_case.py $case > $O/${tool}_${case}.log 2>&1
     echo "$tool $case rc=$?" | tee -a $O/summary.txt

@@ -17,7 +17,7 @@ import vbgen  # noqa: E402
 import paper_conf_ipps_abdelfattahhtd16_b200 as vb  # noqa: E402
 from harness import DeviceBatch  # noqa: E402
 
-KIND = {30: "blocked", 20: "small", 21: "small_la", 22: "small_la2", 40: "warp"}
+KIND = {30: "blocked", 20: "small", 21: "small_la", 22: "small_la2", 23: "quad", 40: "warp"}
 L = vb.lib()
 L.vbatched_debug_timeline.argtypes = [ctypes.c_void_p]
 
