@@ -59,6 +59,11 @@ def lib():
                                    ctypes.c_int, ctypes.c_double, _dp, ctypes.c_int, _dp, ctypes.c_int]
         L.oracle_backward_error.argtypes = [ctypes.c_int, _dp, ctypes.c_int, _dp, ctypes.c_int, ctypes.c_int]
         L.oracle_backward_error.restype = ctypes.c_double
+        L.oracle_dgetrf.argtypes = [ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int, _ip]
+        L.oracle_dgetrf.restype = ctypes.c_int
+        L.oracle_getrf_backward_error.argtypes = [ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int, _dp,
+                                                  ctypes.c_int, _ip]
+        L.oracle_getrf_backward_error.restype = ctypes.c_double
         L.oracle_backward_error_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip,
                                                   ctypes.POINTER(_dp), _ip, _ip, _dp, ctypes.c_int]
         _lib = L
@@ -201,3 +206,27 @@ def rowscaled_diff(Lg: np.ndarray, Lo: np.ndarray, nb: int) -> float:
     rn = np.sqrt(np.sum(o * o, axis=1))
     rn[rn == 0] = 1.0
     return float(np.max(np.abs(g - o) / rn[:, None]))
+
+
+def dgetrf(a: np.ndarray) -> tuple[np.ndarray, np.ndarray, int]:
+    """Oracle LU with partial pivoting of one m x n matrix (oracle.c: textbook unblocked
+    elimination, LAPACK DGETF2 conventions). Returns (factored copy: L strictly below the
+    diagonal, U on/above; ipiv (1-based, int32, min(m,n)); info)."""
+    out = np.array(a, dtype=np.float64, order="F", copy=True)
+    m, n = out.shape
+    ipiv = np.zeros(max(1, min(m, n)), dtype=np.int32)
+    info = lib().oracle_dgetrf(m, n, _ptr(out), max(1, m), ipiv.ctypes.data_as(_ip))
+    return out, ipiv[: min(m, n)], info
+
+
+def getrf_backward_error(A0: np.ndarray, F: np.ndarray, ipiv: np.ndarray) -> float:
+    """||P A - L U||_F / (max(m,n) ||A||_F 2^-53) in long double (L unit lower from F's strict
+    lower part, U = F's upper part, P from ipiv applied in order)."""
+    A0 = np.asfortranarray(A0, dtype=np.float64)
+    F = np.asfortranarray(F, dtype=np.float64)
+    m, n = A0.shape
+    ip = np.ascontiguousarray(ipiv, dtype=np.int32)
+    if ip.size == 0:
+        ip = np.zeros(1, np.int32)
+    return lib().oracle_getrf_backward_error(m, n, _ptr(A0), max(1, m), _ptr(F), max(1, F.shape[0]),
+                                             ip.ctypes.data_as(_ip))

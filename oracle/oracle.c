@@ -29,6 +29,13 @@
  *    kernels (§III-E: potf2, trsm, gemm, syrk), as plain loops.
  *  - oracle_backward_error: ||A - L L^T||_F / (n ||A||_F eps) in long double
  *    (BASELINE.json north_star gate; SURVEY.md §8(c) reading #13, eps = 2^-53).
+ *  - oracle_dgetrf: LU with partial pivoting, A = P L U (the extension to LU the paper names
+ *    as future work, §V, and PAPER.md:740-744, §III-E; SURVEY.md §8(f)
+ *    NEXT-4). Written as the textbook unblocked right-looking elimination with LAPACK DGETF2
+ *    conventions: pivot = first row of maximal |a_ik| (IDAMAX), row swap, l_ik = a_ik / u_kk
+ *    (IEEE division), rank-1 update a_ij -= l_ik u_kj in k order; a zero pivot records
+ *    info = k+1 (first only) and elimination continues (nothing to scale: the column is zero).
+ *  - oracle_getrf_backward_error: ||P A - L U||_F / (max(m,n) ||A||_F eps), long double.
  */
 #include <math.h>
 #include <stdlib.h>
@@ -269,4 +276,79 @@ void oracle_backward_error_batch(int batch, const int* n, double* const* A0, con
 #endif
   for (int b = 0; b < batch; ++b)
     out[b] = oracle_backward_error(n[b], A0[b], lda0[b], Lf[b], ldl[b], info[b]);
+}
+
+/* LU with partial pivoting of the m x n column-major a (leading dim lda), in place: on return
+ * the strict lower part holds L (unit diagonal not stored), the upper part U; ipiv[k] (1-based)
+ * is the row interchanged with row k (k < min(m,n)). Returns LAPACK info (0, or the 1-based
+ * index of the first exactly-zero pivot). */
+int oracle_dgetrf(int m, int n, double* a, int lda, int* ipiv) {
+  const int kmax = m < n ? m : n;
+  int info = 0;
+  for (int k = 0; k < kmax; ++k) {
+    int p = k;
+    double best = fabs(a[IDX(k, k, lda)]);
+    for (int i = k + 1; i < m; ++i) {
+      const double v = fabs(a[IDX(i, k, lda)]);
+      if (v > best) { best = v; p = i; }
+    }
+    ipiv[k] = p + 1;
+    if (a[IDX(p, k, lda)] != 0.0) {
+      if (p != k)
+        for (int j = 0; j < n; ++j) {
+          const double t = a[IDX(k, j, lda)];
+          a[IDX(k, j, lda)] = a[IDX(p, j, lda)];
+          a[IDX(p, j, lda)] = t;
+        }
+      const double piv = a[IDX(k, k, lda)];
+      for (int i = k + 1; i < m; ++i) a[IDX(i, k, lda)] = a[IDX(i, k, lda)] / piv;
+    } else if (info == 0) {
+      info = k + 1;
+    }
+    for (int j = k + 1; j < n; ++j) {
+      const double ukj = a[IDX(k, j, lda)];
+      for (int i = k + 1; i < m; ++i) a[IDX(i, j, lda)] = a[IDX(i, j, lda)] - a[IDX(i, k, lda)] * ukj;
+    }
+  }
+  return info;
+}
+
+/* ||P A - L U||_F / (max(m,n) ||A||_F eps), eps = 2^-53, long double. A0: the original m x n
+ * matrix; F: the factored one (L strictly below the diagonal, unit diagonal implied; U on and
+ * above); ipiv as returned by DGETRF. P A is formed by applying the interchanges in order. */
+double oracle_getrf_backward_error(int m, int n, const double* A0, int lda0, const double* F,
+                                   int ldf, const int* ipiv) {
+  const int kmax = m < n ? m : n;
+  if (m <= 0 || n <= 0) return 0.0;
+  long double* PA = (long double*)malloc(sizeof(long double) * (size_t)m * (size_t)n);
+  for (int j = 0; j < n; ++j)
+    for (int i = 0; i < m; ++i) PA[(size_t)j * m + i] = (long double)A0[IDX(i, j, lda0)];
+  for (int k = 0; k < kmax; ++k) {
+    const int p = ipiv[k] - 1;
+    if (p != k)
+      for (int j = 0; j < n; ++j) {
+        const long double t = PA[(size_t)j * m + k];
+        PA[(size_t)j * m + k] = PA[(size_t)j * m + p];
+        PA[(size_t)j * m + p] = t;
+      }
+  }
+  long double num = 0.0L, den = 0.0L;
+  for (int j = 0; j < n; ++j)
+    for (int i = 0; i < m; ++i) {
+      long double s = 0.0L;
+      const int kk = (i < j ? i : j) < kmax ? (i < j ? i : j) : kmax - 1;
+      for (int k = 0; k <= kk && k < kmax; ++k) {
+        const long double l = (i == k) ? 1.0L : (i > k ? (long double)F[IDX(i, k, ldf)] : 0.0L);
+        const long double u = (k <= j) ? (long double)F[IDX(k, j, ldf)] : 0.0L;
+        s += l * u;
+      }
+      const long double d = PA[(size_t)j * m + i] - s;
+      num += d * d;
+      den += PA[(size_t)j * m + i] * PA[(size_t)j * m + i];
+    }
+  free(PA);
+  if (den == 0.0L) return num == 0.0L ? 0.0 : INFINITY;
+  const long double eps = ldexpl(1.0L, -53);
+  const int mx = m > n ? m : n;
+  return (double)(sqrtl(num) / ((long double)mx * sqrtl(den) * eps));
 }

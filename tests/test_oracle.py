@@ -557,3 +557,139 @@ def test_rowscaled_gate_closed_form():
     Ln = Lo.copy()
     Ln[2, 1] = np.nan
     assert not (oracle.rowscaled_diff(Ln, Lo, 4) <= 1e-10)
+
+
+# ---------------------------------------------------------------- LU
+def _apply_ipiv(A, ipiv):
+    """P A for LAPACK interchanges ipiv (1-based), applied in order."""
+    B = np.array(A, dtype=np.float64, copy=True)
+    for k, p in enumerate(ipiv):
+        if p - 1 != k:
+            B[[k, p - 1], :] = B[[p - 1, k], :]
+    return B
+
+
+def _split_lu(F):
+    m, n = F.shape
+    k = min(m, n)
+    L = np.tril(F[:, :k], -1) + np.eye(m, k)
+    U = np.triu(F[:k, :])
+    return L, U
+
+
+def test_lu_handworked_golden():
+    g = json.load(open(os.path.join(GOLD, "lu_handworked.json")))
+    for c in g["cases"]:
+        F, ipiv, info = oracle.dgetrf(np.array(c["A"], dtype=np.float64))
+        assert np.array_equal(F, np.array(c["F"], dtype=np.float64)), c["name"]
+        assert list(ipiv) == c["ipiv"] and info == c["info"], c["name"]
+
+
+@pytest.mark.parametrize("m,n", [(1, 1), (5, 5), (33, 33), (64, 40), (40, 64), (130, 130)])
+def test_lu_exact_family(m, n):
+    """A = P0 L U with unit-lower L (|l_ik| <= 1/2, dyadic) and integer U whose pivots dominate:
+    partial pivoting must select exactly the rows P0 moved, and L, U come back bit-exactly."""
+    rng = np.random.default_rng(1000 + 7 * m + n)
+    k = min(m, n)
+    L = np.tril(rng.choice([-0.5, -0.25, 0.0, 0.25, 0.5], size=(m, k)), -1) + np.eye(m, k)
+    U = np.triu(rng.integers(-3, 4, size=(k, n)).astype(np.float64), 1)
+    U[np.arange(k), np.arange(k)] = rng.choice([-8.0, -4.0, 4.0, 8.0], size=k)
+    A = L @ U  # exact: dyadic products, small sums
+    perm = rng.permutation(m)
+    A0 = A[perm]
+    F, ipiv, info = oracle.dgetrf(A0)
+    assert info == 0
+    Lg, Ug = _split_lu(F)
+    assert np.array_equal(Ug, U)
+    # the k pivot rows are A's first k rows in order (their l = 1 entries dominate), so L's top
+    # k rows come back exactly; the rows below are a row permutation of L's (order set by the
+    # interchanges), and P A0 = L U holds bit-exactly
+    assert np.array_equal(Lg[:k], L[:k])
+    key = lambda M: M[np.lexsort(M.T[::-1])]  # noqa: E731
+    assert np.array_equal(key(Lg[k:]), key(L[k:]))
+    assert np.array_equal(_apply_ipiv(A0, ipiv), Lg @ Ug)
+
+
+@pytest.mark.parametrize("m,n", [(7, 7), (64, 64), (100, 37), (37, 100), (257, 257)])
+def test_lu_matches_lapack(m, n):
+    """ipiv bit-exact and the factors within 1e-12 of LAPACK DGETRF (OpenBLAS via scipy, MKL via
+    torch) on the general random family."""
+    import scipy.linalg
+    import torch
+    A = vbgen.g1_matrix(11, m * 1000 + n, m, n)
+    F, ipiv, info = oracle.dgetrf(A)
+    lu, piv = scipy.linalg.lu_factor(A, check_finite=False)
+    k = min(m, n)
+    assert info == 0
+    assert np.array_equal(ipiv, (piv[:k] + 1).astype(np.int32))
+    assert np.max(np.abs(F - lu)) <= 1e-12 * max(1.0, np.max(np.abs(lu)))
+    LU_t, piv_t = torch.linalg.lu_factor(torch.from_numpy(np.array(A)))
+    assert np.array_equal(ipiv, piv_t.numpy()[:k].astype(np.int32))
+    assert np.max(np.abs(F - LU_t.numpy())) <= 1e-12 * max(1.0, np.max(np.abs(lu)))
+
+
+def test_lu_singular_info():
+    A = np.ones((6, 6))
+    _, _, info = oracle.dgetrf(A)
+    assert info == 2  # second pivot exactly zero (rows all equal)
+    B = vbgen.g1_matrix(3, 5, 8, 8)
+    B[:, 3] = 0.0
+    _, ipiv, info = oracle.dgetrf(B)
+    assert info == 4 and ipiv[3] == 4  # zero column: no interchange, info = first zero pivot
+    Z = np.zeros((3, 5))
+    F, ipiv, info = oracle.dgetrf(Z)
+    assert info == 1 and list(ipiv) == [1, 2, 3] and not F.any()
+
+
+def test_lu_det_invariant_exact_rational():
+    """det(A) = (-1)^(#swaps) prod u_kk, against an exact rational determinant (Bareiss-free
+    Fraction elimination) of small integer matrices."""
+    rng = np.random.default_rng(77)
+    for n in (2, 3, 5, 8):
+        A = rng.integers(-9, 10, size=(n, n)).astype(np.float64)
+        M = [[Fraction(int(x)) for x in row] for row in A]
+        det = Fraction(1)
+        for k in range(n):
+            p = next((i for i in range(k, n) if M[i][k] != 0), None)
+            if p is None:
+                det = Fraction(0)
+                break
+            if p != k:
+                M[k], M[p] = M[p], M[k]
+                det = -det
+            det *= M[k][k]
+            for i in range(k + 1, n):
+                f = M[i][k] / M[k][k]
+                for j in range(k, n):
+                    M[i][j] -= f * M[k][j]
+        F, ipiv, info = oracle.dgetrf(A)
+        sign = (-1) ** sum(1 for k, p in enumerate(ipiv) if p - 1 != k)
+        got = sign * np.prod(np.diag(F))
+        assert got == pytest.approx(float(det), rel=1e-12, abs=1e-12)
+
+
+def test_lu_backward_error_gate_closed_form():
+    """oracle_getrf_backward_error: 0 on an exact factorisation; equals the Fraction closed form
+    ||P A - L U||_F / (max(m,n) ||A||_F 2^-53) for a known perturbation of U; dgetrf's own
+    factors of a random matrix stay far below 10."""
+    m, n = 6, 4
+    rng = np.random.default_rng(5)
+    L = np.tril(rng.choice([-0.5, 0.25, 0.5], size=(m, n)), -1) + np.eye(m, n)
+    U = np.triu(rng.integers(-3, 4, size=(n, n)).astype(np.float64), 1) + np.diag([8.0, -8, 4, 4])
+    A = L @ U
+    F, ipiv, info = oracle.dgetrf(A)
+    assert info == 0 and oracle.getrf_backward_error(A, F, ipiv) == 0.0
+    F2 = F.copy(order="F")
+    F2[1, 2] += 2.0 ** -30
+    Lf, Uf = _split_lu(F2)
+    PA = [[Fraction(float(x)) for x in row] for row in _apply_ipiv(A, ipiv)]
+    LfF = [[Fraction(float(x)) for x in row] for row in Lf]
+    UfF = [[Fraction(float(x)) for x in row] for row in Uf]
+    num = sum((PA[i][j] - sum((LfF[i][k] * UfF[k][j] for k in range(n)), Fraction(0))) ** 2
+              for i in range(m) for j in range(n))
+    den = sum(x * x for row in PA for x in row)
+    exp = math.sqrt(num) / (max(m, n) * math.sqrt(den) * 2.0 ** -53)
+    assert oracle.getrf_backward_error(A, F2, ipiv) == pytest.approx(exp, rel=1e-9)
+    G = vbgen.g1_matrix(2, 9, 200, 200)
+    FG, ipg, _ = oracle.dgetrf(G)
+    assert oracle.getrf_backward_error(G, FG, ipg) < 10

@@ -124,6 +124,21 @@ def f2_matrix(seed: int, gidx: int, n: int, kappa: float = 1e4) -> np.ndarray:
     return np.asfortranarray((A + A.T) / 2)
 
 
+def g1_matrix(seed: int, gidx: int, m: int, n: int) -> np.ndarray:
+    """General (non-symmetric) m x n matrix for the LU path: a_ij =
+    2 u(seed, gidx, i, j) - 1 in [-1, 1) from the same counter hash, keyed by (i, j) — no
+    symmetry. Input generation only."""
+    if m == 0 or n == 0:
+        return np.zeros((m, n), order="F")
+    i = np.arange(m)[:, None] + np.zeros((1, n), np.int64)
+    j = np.arange(n)[None, :] + np.zeros((m, 1), np.int64)
+    key = (np.uint64(gidx) << np.uint64(42)) ^ (i.astype(np.uint64) << np.uint64(21)) ^ \
+        j.astype(np.uint64) ^ np.uint64(0x1 << 63)
+    h = splitmix64(splitmix64(np.uint64(seed)) ^ key)
+    u = (h >> np.uint64(11)).astype(np.float64) * (2.0 ** -53)
+    return np.asfortranarray(2.0 * u - 1.0)
+
+
 def config_matrix(cfg: Config | str, gidx: int, n: int | None = None) -> np.ndarray:
     if isinstance(cfg, str):
         cfg = CONFIGS[cfg]
