@@ -144,3 +144,80 @@ def gpu_backward_errors(db: DeviceBatch, chunk_elems: int = 1 << 26) -> np.ndarr
             den = torch.linalg.matrix_norm(A)
             out[ii] = (num / (n * den * eps)).cpu().numpy()
     return out
+
+
+class LUBatch:
+    """A vbatched general-matrix problem for vbatched_dgetrf: arena of m_i x n_i column-major
+    matrices (leading dims ldda_i, 256 B aligned), ipiv arena (min(m,n) int32 per matrix) and
+    the device pointer arrays. Values: vbgen.g1_matrix(seed, gidx, m, n) unless set."""
+
+    def __init__(self, m, n, seed=1, ldda=None, device="cuda"):
+        self.m = np.ascontiguousarray(m, dtype=np.int32)
+        self.n = np.ascontiguousarray(n, dtype=np.int32)
+        self.B = len(self.m)
+        self.seed = seed
+        self.ldda = np.ascontiguousarray(np.maximum(1, self.m) if ldda is None else ldda, dtype=np.int32)
+        self.off, total = vbgen.arena_layout(np.maximum(self.n, 0), self.ldda)
+        self.arena = torch.full((total,), float("nan"), dtype=torch.float64, device=device)
+        k = np.maximum(0, np.minimum(self.m, self.n)).astype(np.int64)
+        self.ioff = np.concatenate([[0], np.cumsum((k + 63) // 64 * 64)[:-1]]).astype(np.int64)
+        self.ipiv = torch.full((int(self.ioff[-1] + max(64, k[-1] + 64)),), -7, dtype=torch.int32,
+                               device=device)
+        self.d_ptrs = torch.from_numpy((self.arena.data_ptr() + 8 * self.off).astype(np.int64)).to(device)
+        self.d_ipiv = torch.from_numpy((self.ipiv.data_ptr() + 4 * self.ioff).astype(np.int64)).to(device)
+        self.d_m = torch.from_numpy(self.m).to(device)
+        self.d_n = torch.from_numpy(self.n).to(device)
+        self.d_ldda = torch.from_numpy(self.ldda).to(device)
+        self.d_info = torch.full((max(self.B, 1),), -12345, dtype=torch.int32, device=device)
+        self.inputs = {}
+
+    def set_matrix(self, i, A):
+        m, n, ld = int(self.m[i]), int(self.n[i]), int(self.ldda[i])
+        blk = np.full((ld, n), np.nan)
+        blk.view(np.uint64)[:] = np.uint64(vbgen.NAN_POISON_BITS)
+        blk[:m, :] = A
+        self.inputs[i] = np.asfortranarray(A)
+        self.arena[self.off[i]: self.off[i] + ld * n].copy_(torch.from_numpy(blk.ravel(order="F").copy()))
+
+    def fill(self):
+        for i in range(self.B):
+            if self.m[i] > 0 and self.n[i] > 0:
+                self.set_matrix(i, vbgen.g1_matrix(self.seed, i, int(self.m[i]), int(self.n[i])))
+        return self
+
+    def getrf(self, max_m=None, max_n=None, stream=None, check=True):
+        from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dgetrf
+        mm = int(self.m.max()) if max_m is None else max_m
+        mn = int(self.n.max()) if max_n is None else max_n
+        return vbatched_dgetrf(self.d_m, self.d_n, self.d_ptrs, self.d_ldda, self.d_ipiv, self.d_info,
+                               self.B, mm, mn, stream=stream, check=check)
+
+    def block(self, i):
+        m, n, ld = int(self.m[i]), int(self.n[i]), int(self.ldda[i])
+        return self.arena[self.off[i]: self.off[i] + ld * n].cpu().numpy().reshape((ld, n), order="F")
+
+    def ipiv_of(self, i):
+        k = max(0, min(int(self.m[i]), int(self.n[i])))
+        return self.ipiv[int(self.ioff[i]): int(self.ioff[i]) + k].cpu().numpy()
+
+    def info(self):
+        return self.d_info[: self.B].cpu().numpy()
+
+
+def compare_lu_with_oracle(A_in, F_gpu, ipiv_gpu, info_gpu):
+    """LU parity gates (SURVEY.md §8(f) NEXT-4; DESIGN.md readings): info and ipiv bit-exact;
+    backward error ||P A - L U||_F / (max(m,n) ||A||_F eps) <= 10; every entry of the factored
+    matrix within 1e-10 of the oracle's, scaled by the norm of the oracle's row."""
+    import oracle
+    m, n = A_in.shape
+    Fo, ipo, info_o = oracle.dgetrf(A_in)
+    Fg = np.asfortranarray(F_gpu[:m, :n])
+    res = {"m": m, "n": n, "info_oracle": info_o, "info_gpu": int(info_gpu),
+           "ipiv_equal": bool(np.array_equal(np.asarray(ipiv_gpu), ipo))}
+    res["bwd"] = oracle.getrf_backward_error(A_in, Fg, np.asarray(ipiv_gpu, np.int32)) if m and n else 0.0
+    rn = np.sqrt(np.sum(Fo * Fo, axis=1))
+    rn[rn == 0] = 1.0
+    res["rowscaled"] = float(np.max(np.abs(Fg - Fo) / rn[:, None])) if m and n else 0.0
+    res["ok"] = (res["info_oracle"] == res["info_gpu"] and res["ipiv_equal"] and res["bwd"] <= 10.0
+                 and res["rowscaled"] <= 1e-10)
+    return res

@@ -187,6 +187,31 @@ int vbatched_dposv(char uplo, const int* d_n, const int* d_nrhs, double* const* 
                    int batchCount, int max_n, int max_nrhs, vb_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------
+ * vbatched_dgetrf — FP64 variable-size batched LU with partial pivoting, A_i = P_i L_i U_i
+ * (the LU extension the paper names as future work, PAPER.md:2279-2285
+ * §V, built from its vbatched kernels, §III-E; LAPACK DGETRF semantics).
+ *
+ *  d_m, d_n     [batchCount] rows m_i and columns n_i (device). Rectangular matrices allowed.
+ *  dA_array     [batchCount] device pointers; A_i is m_i x n_i column-major with leading
+ *               dimension d_ldda[i] >= max(1, m_i). On return: L_i strictly below the diagonal
+ *               (unit diagonal not stored), U_i on and above it. Rows m_i..ldda_i-1 untouched.
+ *  dipiv_array  [batchCount] device pointers to int arrays of min(m_i, n_i) entries: row k was
+ *               interchanged with row ipiv[k] (1-based, LAPACK convention), in order.
+ *  d_info       [batchCount] output: 0; k > 0 = U(k,k) is exactly zero (first such k, 1-based;
+ *               the factorisation is completed, as LAPACK DGETRF); -1 m_i < 0; -2 n_i < 0;
+ *               -4 ldda_i < max(1, m_i); -9 m_i > max_m or n_i > max_n (matrix untouched).
+ *  max_m, max_n upper bounds on every m_i / n_i (host). max_m <= 1024 (the panel rows are held
+ *               in registers): larger returns -8.
+ * Pivot: the first row of maximal |a_ik| (IDAMAX). Arithmetic: panel (16 columns) in registers
+ * with IEEE division for the multipliers, then the library's vbatched DTRSM (side L, lower,
+ * unit) and DGEMM (DMMA) on the trailing matrix, one panel step at a time (PAPER.md:724-812,
+ * the separated design). Returns 0 / -p (batchCount -7, max_m -8, max_n -9) / cudaError_t.
+ */
+int vbatched_dgetrf(const int* d_m, const int* d_n, double* const* dA_array, const int* d_ldda,
+                    int* const* dipiv_array, int* d_info, int batchCount, int max_m, int max_n,
+                    vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
  * Host helpers (pure host, deterministic, no CUDA).
  * vbatched_partition_lpt: flop-balanced multi-GPU sharding: longest
  *   processing time first on cost n^3/3 — sort by n descending (ties by index), assign

@@ -20,7 +20,7 @@ __all__ = [
     "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
     "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "vbatched_dpotrf_kernel_names",
-    "vbatched_release_host_staging", "factor_kernel_names", "lib", "LIB_PATH", "VBatchedError",
+    "vbatched_release_host_staging", "factor_kernel_names", "vbatched_dgetrf", "lib", "LIB_PATH", "VBatchedError",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -68,6 +68,7 @@ def lib() -> ctypes.CDLL:
         L.vbatched_dpotrf_kernel_launches.restype = _i
         L.vbatched_dpotrf_kernel_names.argtypes = [_i]
         L.vbatched_dpotrf_kernel_names.restype = ctypes.c_char_p
+        L.vbatched_dgetrf.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_release_host_staging.argtypes = []
         L.vbatched_release_host_staging.restype = _i
         L.vbatched_host_alloc.argtypes = [ctypes.c_size_t]
@@ -207,6 +208,15 @@ def vbatched_dposv(uplo, n, nrhs, dA_array, ldda, dB_array, lddb, info, batchCou
                               _ptr(dB_array), _ptr(lddb), _ptr(info), int(batchCount), int(max_n),
                               int(max_nrhs), _stream(stream))
     return _check(rc, "vbatched_dposv") if check else rc
+
+
+def vbatched_dgetrf(m, n, dA_array, ldda, dipiv_array, info, batchCount, max_m, max_n, stream=None,
+                    check=True):
+    """vbatched LU with partial pivoting (include/vbatched.h): device arrays m, n, ldda, info
+    (int32), dA_array / dipiv_array (int64 device pointers)."""
+    rc = lib().vbatched_dgetrf(_ptr(m), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(dipiv_array),
+                               _ptr(info), int(batchCount), int(max_m), int(max_n), _stream(stream))
+    return _check(rc, "vbatched_dgetrf") if check else rc
 
 
 def vbatched_partition_lpt(h_n, ngpu: int):

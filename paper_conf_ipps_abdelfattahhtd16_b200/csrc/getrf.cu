@@ -1,0 +1,295 @@
+// getrf.cu — vbatched LU with partial pivoting (DGETRF): the extension
+// to LU that the paper names as future work ("the extension of this work to the LU and QR
+// factorizations ... where many of the BLAS kernels proposed here can be reused out of the
+// box", §V; "these kernels are a foundation for other variable-size batched
+// factorizations (LU and QR)", §III-E).
+//
+// Built the paper's "separated" way: a host loop over panels of NB columns,
+// each step = an aux kernel that derives the per-matrix sub-problem sizes and pointers on the
+// GPU (the size arrays live there), a fused panel kernel (getf2 with partial
+// pivoting, rows in registers), the row interchanges on the other columns (laswp), and then
+// the SAME vbatched TRSM and GEMM kernels that vbatched_dtrsm / vbatched_dgemm export:
+//   A12 <- L11^-1 A12   (vbatched TRSM, side L, lower, unit diagonal)
+//   A22 <- A22 - A21 A12 (vbatched GEMM, DMMA)
+// Matrices whose panel is exhausted get size 0 in the step arrays and cost no tiles.
+#include <algorithm>
+
+#include "../../include/vbatched.h"
+#include "common.cuh"
+#include "internal.h"
+
+namespace vb {
+namespace {
+
+constexpr int kLuNB = 16;        // panel width
+constexpr int kLuThreads = 256;  // panel kernel CTA
+constexpr int kLuMaxRPT = 4;     // rows per thread held in registers: m - j <= 1024
+
+struct LuStep {
+  int* pm;   // panel rows (m_i - j), 0 when the matrix has no panel at step j
+  int* pn;   // panel width (<= NB)
+  int* rn;   // columns right of the panel
+  int* bm;   // rows below the panel
+  double** P;    // panel top-left A_i(j, j)
+  double** A12;  // A_i(j, j + pn)
+  double** A21;  // A_i(j + pn, j)
+  double** A22;  // A_i(j + pn, j + pn)
+};
+
+// info: -1 m < 0, -2 n < 0, -4 ldda < max(1, m), -9 m > max_m or n > max_n; else 0.
+__global__ void lu_validate_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                                   const int* __restrict__ d_ld, int* __restrict__ d_info, int batch,
+                                   int max_m, int max_n) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    int code = 0;
+    if (m < 0) code = -1;
+    else if (n < 0) code = -2;
+    else if (ld < (m > 1 ? m : 1)) code = -4;
+    else if (m > max_m || n > max_n) code = -9;
+    d_info[i] = code;
+  }
+}
+
+__global__ void lu_step_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                               double* const* __restrict__ dA, const int* __restrict__ d_ld,
+                               const int* __restrict__ d_info, int batch, int j, LuStep st) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    const int kmax = m < n ? m : n;
+    const bool act = d_info[i] >= 0 && j < kmax;
+    const int nb = act ? min(kLuNB, kmax - j) : 0;
+    st.pm[i] = act ? m - j : 0;
+    st.pn[i] = nb;
+    st.rn[i] = act ? n - j - nb : 0;
+    st.bm[i] = act ? m - j - nb : 0;
+    double* A = dA[i];
+    st.P[i] = act ? A + (size_t)j * ld + j : A;
+    st.A12[i] = act ? A + (size_t)(j + nb) * ld + j : A;
+    st.A21[i] = act ? A + (size_t)j * ld + j + nb : A;
+    st.A22[i] = act ? A + (size_t)(j + nb) * ld + j + nb : A;
+  }
+}
+
+// Panel factorisation with partial pivoting (LAPACK DGETF2 on the pm x pn panel): one CTA per
+// matrix, thread t holds rows t, t + 256, ... (RPT of them) x NB columns in registers. Column k:
+// block argmax of |a_rk| over rows r >= k (ties -> smallest row, as IDAMAX), the pivot row and
+// row k trade places through shared memory, l_rk = a_rk / u_kk (IEEE division), rank-1 update
+// of the panel's later columns. A zero pivot (the whole column is zero) records info = j+k+1
+// (first only) and is skipped, as in DGETF2. ipiv gets the global 1-based interchanges.
+template <int RPT>
+__global__ void __launch_bounds__(kLuThreads)
+    lu_panel_kernel(LuStep st, const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv,
+                    int* __restrict__ d_info, int batch, int j) {
+  __shared__ double prow[kLuNB], krow[kLuNB];
+  __shared__ double wval[kLuThreads / 32];
+  __shared__ int wrow[kLuThreads / 32];
+  __shared__ int s_piv, s_zero;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = blockIdx.x; i < batch; i += gridDim.x) {
+    const int pm = st.pm[i], pn = st.pn[i];
+    if (pm <= 0 || pn <= 0) continue;
+    const int ld = d_ld[i];
+    double* P = st.P[i];
+    double a[RPT][kLuNB];
+#pragma unroll
+    for (int s = 0; s < RPT; ++s) {
+      const int r = tid + s * kLuThreads;
+#pragma unroll
+      for (int c = 0; c < kLuNB; ++c) a[s][c] = (r < pm && c < pn) ? P[(size_t)c * ld + r] : 0.0;
+    }
+    if (tid == 0) s_zero = -1;
+#pragma unroll
+    for (int k = 0; k < kLuNB; ++k) {
+      if (k >= pn) break;
+      // ---- pivot search: first row of maximal |a_rk|, r >= k
+      double best = -1.0;
+      int brow = 0x7fffffff;
+#pragma unroll
+      for (int s = 0; s < RPT; ++s) {
+        const int r = tid + s * kLuThreads;
+        const double v = fabs(a[s][k]);
+        if (r >= k && r < pm && v > best) {
+          best = v;
+          brow = r;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        const double ov = __shfl_xor_sync(kFull, best, o);
+        const int orow = __shfl_xor_sync(kFull, brow, o);
+        if (ov > best || (ov == best && orow < brow)) {
+          best = ov;
+          brow = orow;
+        }
+      }
+      if (lane == 0) {
+        wval[warp] = best;
+        wrow[warp] = brow;
+      }
+      __syncthreads();
+      if (tid == 0) {
+        double bv = wval[0];
+        int br = wrow[0];
+        for (int w = 1; w < kLuThreads / 32; ++w)
+          if (wval[w] > bv || (wval[w] == bv && wrow[w] < br)) {
+            bv = wval[w];
+            br = wrow[w];
+          }
+        s_piv = br;
+        d_ipiv[i][j + k] = j + br + 1;
+      }
+      __syncthreads();
+      const int p = s_piv;
+      // ---- the pivot row and row k trade places (through shared memory)
+#pragma unroll
+      for (int s = 0; s < RPT; ++s) {
+        const int r = tid + s * kLuThreads;
+        if (r == p)
+#pragma unroll
+          for (int c = 0; c < kLuNB; ++c) prow[c] = a[s][c];
+        if (r == k)
+#pragma unroll
+          for (int c = 0; c < kLuNB; ++c) krow[c] = a[s][c];
+      }
+      __syncthreads();
+      const double piv = prow[k];
+#pragma unroll
+      for (int s = 0; s < RPT; ++s) {
+        const int r = tid + s * kLuThreads;
+        if (r == k)
+#pragma unroll
+          for (int c = 0; c < kLuNB; ++c) a[s][c] = prow[c];
+        else if (r == p)
+#pragma unroll
+          for (int c = 0; c < kLuNB; ++c) a[s][c] = krow[c];
+      }
+      if (piv != 0.0) {
+#pragma unroll
+        for (int s = 0; s < RPT; ++s) {
+          const int r = tid + s * kLuThreads;
+          if (r > k && r < pm) {
+            const double l = a[s][k] / piv;
+            a[s][k] = l;
+#pragma unroll
+            for (int c = k + 1; c < kLuNB; ++c) a[s][c] = fma(-l, prow[c], a[s][c]);
+          }
+        }
+      } else if (tid == 0 && s_zero < 0) {
+        s_zero = k;
+      }
+      __syncthreads();  // prow/krow/wval are rewritten by the next column
+    }
+#pragma unroll
+    for (int s = 0; s < RPT; ++s) {
+      const int r = tid + s * kLuThreads;
+      if (r < pm)
+#pragma unroll
+        for (int c = 0; c < kLuNB; ++c)
+          if (c < pn) P[(size_t)c * ld + r] = a[s][c];
+    }
+    if (tid == 0 && s_zero >= 0 && d_info[i] == 0) d_info[i] = j + s_zero + 1;
+    __syncthreads();
+  }
+}
+
+// Row interchanges of the step's pivots on the columns outside the panel (LAPACK DLASWP on
+// columns 0..j-1 and j+pn..n-1): one CTA per matrix, a thread per column, pivots in order.
+__global__ void __launch_bounds__(256)
+    lu_laswp_kernel(LuStep st, double* const* __restrict__ dA, const int* __restrict__ d_n,
+                    const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv, int batch, int j) {
+  for (int i = blockIdx.x; i < batch; i += gridDim.x) {
+    const int pn = st.pn[i];
+    if (pn <= 0) continue;
+    const int n = d_n[i], ld = d_ld[i];
+    double* A = dA[i];
+    const int* ip = d_ipiv[i] + j;
+    for (int c = threadIdx.x; c < n; c += blockDim.x) {
+      if (c >= j && c < j + pn) continue;
+      double* col = A + (size_t)c * ld;
+      for (int k = 0; k < pn; ++k) {
+        const int r2 = ip[k] - 1, r1 = j + k;
+        if (r2 != r1) {
+          const double t = col[r1];
+          col[r1] = col[r2];
+          col[r2] = t;
+        }
+      }
+    }
+  }
+}
+
+template <int RPT>
+cudaError_t launch_panel(int grid, LuStep st, const int* d_ld, int* const* d_ipiv, int* d_info,
+                         int batch, int j, cudaStream_t stream) {
+  lu_panel_kernel<RPT><<<grid, kLuThreads, 0, stream>>>(st, d_ld, d_ipiv, d_info, batch, j);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+int getrf_impl(const int* d_m, const int* d_n, double* const* dA, const int* d_ld,
+               int* const* d_ipiv, int* d_info, int batch, int max_m, int max_n,
+               cudaStream_t stream) {
+  if (max_m > kLuThreads * kLuMaxRPT) return -8;  // panel rows are held in registers
+  int dev = 0, sms = 148;
+  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  void* ws = nullptr;
+  const size_t ibytes = sizeof(int) * (size_t)batch, pbytes = sizeof(double*) * (size_t)batch;
+  cudaError_t e = ws_alloc(&ws, 4 * ibytes + 4 * pbytes + 64, stream);
+  if (e != cudaSuccess) return (int)e;
+  char* w = static_cast<char*>(ws);
+  LuStep st;
+  st.P = reinterpret_cast<double**>(w);
+  st.A12 = st.P + batch;
+  st.A21 = st.A12 + batch;
+  st.A22 = st.A21 + batch;
+  st.pm = reinterpret_cast<int*>(st.A22 + batch);
+  st.pn = st.pm + batch;
+  st.rn = st.pn + batch;
+  st.bm = st.rn + batch;
+  const int eg = std::max(1, std::min((batch + 255) / 256, 4 * sms));
+  lu_validate_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, d_ld, d_info, batch, max_m, max_n);
+  e = cudaGetLastError();
+  const int kmax = std::min(max_m, max_n);
+  const int pg = std::max(1, std::min(batch, 8 * sms));
+  for (int j = 0; j < kmax && e == cudaSuccess; j += kLuNB) {
+    lu_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, batch, j, st);
+    if ((e = cudaGetLastError()) != cudaSuccess) break;
+    const int rows = max_m - j;
+    if (rows <= kLuThreads) e = launch_panel<1>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+    else if (rows <= 2 * kLuThreads) e = launch_panel<2>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+    else e = launch_panel<4>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+    if (e != cudaSuccess) break;
+    lu_laswp_kernel<<<pg, 256, 0, stream>>>(st, dA, d_n, d_ld, d_ipiv, batch, j);
+    if ((e = cudaGetLastError()) != cudaSuccess) break;
+    if (j + kLuNB < max_n) {
+      int rc = trsm_launch('L', 'L', 'N', 'U', st.pn, st.rn, 1.0, st.P, d_ld, st.A12, d_ld, batch,
+                           kLuNB, max_n, stream);
+      if (rc == 0)
+        rc = gemm_launch('N', 'N', st.bm, st.rn, st.pn, -1.0, st.A21, d_ld, st.A12, d_ld, 1.0,
+                         st.A22, d_ld, batch, max_m, max_n, kLuNB, stream);
+      if (rc != 0) {
+        e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
+        break;
+      }
+    }
+  }
+  cudaError_t e2 = ws_free(ws, stream);
+  return (int)(e != cudaSuccess ? e : e2);
+}
+
+}  // namespace vb
+
+using namespace vb;
+
+extern "C" int vbatched_dgetrf(const int* d_m, const int* d_n, double* const* dA_array,
+                               const int* d_ldda, int* const* dipiv_array, int* d_info,
+                               int batchCount, int max_m, int max_n, vb_stream_t stream) {
+  if (batchCount < 0) return -7;
+  if (max_m < 0) return -8;
+  if (max_n < 0) return -9;
+  if (batchCount == 0) return 0;
+  return getrf_impl(d_m, d_n, dA_array, d_ldda, dipiv_array, d_info, batchCount, max_m, max_n,
+                    (cudaStream_t)stream);
+}
