@@ -221,3 +221,81 @@ def compare_lu_with_oracle(A_in, F_gpu, ipiv_gpu, info_gpu):
     res["ok"] = (res["info_oracle"] == res["info_gpu"] and res["ipiv_equal"] and res["bwd"] <= 10.0
                  and res["rowscaled"] <= 1e-10)
     return res
+
+
+class ZBatch:
+    """A vbatched complex Hermitian problem for vbatched_zpotrf (complex128) / vbatched_cpotrf
+    (complex64): arena of interleaved complex matrices (leading dims ldda, 256 B aligned), the
+    referenced triangle from vbgen.f1c_matrix (or set_matrix), NaN-payload poison elsewhere."""
+
+    def __init__(self, n, seed=1, single=False, ldda=None, nonspd_mod=0, device="cuda"):
+        self.n = np.ascontiguousarray(n, dtype=np.int32)
+        self.B = len(self.n)
+        self.seed, self.single, self.nonspd_mod = seed, single, nonspd_mod
+        self.dt = torch.complex64 if single else torch.complex128
+        self.np_dt = np.complex64 if single else np.complex128
+        es = 8 if single else 16
+        self.ldda = np.ascontiguousarray(np.maximum(1, self.n) if ldda is None else ldda, dtype=np.int32)
+        self.off, total = vbgen.arena_layout(np.maximum(self.n, 0), self.ldda, elem_bytes=es)
+        self.arena = torch.zeros(total, dtype=self.dt, device=device)
+        self.d_ptrs = torch.from_numpy((self.arena.data_ptr() + es * self.off).astype(np.int64)).to(device)
+        self.d_n = torch.from_numpy(self.n).to(device)
+        self.d_ldda = torch.from_numpy(self.ldda).to(device)
+        self.d_info = torch.full((max(self.B, 1),), -12345, dtype=torch.int32, device=device)
+        self.inputs = {}
+
+    def set_matrix(self, i, A, uplo="L"):
+        n, ld = int(self.n[i]), int(self.ldda[i])
+        blk = np.full((ld, n), complex(np.nan, np.nan), dtype=self.np_dt)
+        tri = np.tril(np.ones((n, n), bool)) if uplo == "L" else np.triu(np.ones((n, n), bool))
+        blk[:n, :n] = np.where(tri, np.asarray(A, dtype=self.np_dt), blk[:n, :n])
+        self.inputs[i] = np.asfortranarray(np.asarray(A, dtype=self.np_dt))
+        self.arena[self.off[i]: self.off[i] + ld * n].copy_(torch.from_numpy(blk.ravel(order="F").copy()))
+
+    def fill(self, uplo="L"):
+        for i in range(self.B):
+            if self.n[i] > 0:
+                ns = self.nonspd_mod > 0 and i % self.nonspd_mod == self.nonspd_mod - 1
+                self.set_matrix(i, vbgen.f1c_matrix(self.seed, i, int(self.n[i]), ns), uplo)
+        return self
+
+    def potrf(self, uplo="L", max_n=None, stream=None, check=True):
+        import paper_conf_ipps_abdelfattahhtd16_b200 as vb
+        fn = vb.vbatched_cpotrf if self.single else vb.vbatched_zpotrf
+        mx = int(self.n.max()) if max_n is None else max_n
+        return fn(uplo, self.d_n, self.d_ptrs, self.d_ldda, self.d_info, self.B, mx, stream=stream,
+                  check=check)
+
+    def block(self, i):
+        n, ld = int(self.n[i]), int(self.ldda[i])
+        return self.arena[self.off[i]: self.off[i] + ld * n].cpu().numpy().reshape((ld, n), order="F")
+
+    def info(self):
+        return self.d_info[: self.B].cpu().numpy()
+
+
+def compare_zpotrf_with_oracle(A_in, L_gpu, info_gpu, single=False):
+    """Complex Cholesky gates: info exact; complex backward error <= 10 (eps = 2^-53; FP32
+    storage: the same ratio with eps32, i.e. x 2^-29); row-scaled difference to the oracle's L
+    <= 1e-10 (Z, F1c kappa ~ 1) or 8 n eps32 (C, vs the single-precision oracle)."""
+    import oracle
+    n = A_in.shape[0]
+    if single:
+        Lo, info_o = oracle.cpotrf(A_in.astype(np.complex64))
+    else:
+        Lo, info_o = oracle.zpotrf(A_in)
+    nb = n if info_o == 0 else info_o - 1
+    Lg = np.tril(np.asarray(L_gpu[:n, :n], dtype=np.complex128))
+    res = {"n": n, "info_oracle": info_o, "info_gpu": int(info_gpu)}
+    bwd = oracle.zpotrf_backward_error(np.asarray(A_in, np.complex128), Lg, info_o) if nb else 0.0
+    res["bwd"] = bwd * (2.0 ** -29 if single else 1.0)
+    if nb:
+        o = np.tril(np.asarray(Lo, np.complex128)[:nb, :nb])
+        rn = np.sqrt(np.sum(np.abs(o) ** 2, axis=1))
+        rn[rn == 0] = 1.0
+        res["rowscaled"] = float(np.max(np.abs(Lg[:nb, :nb] - o) / rn[:, None]))
+    else:
+        res["rowscaled"] = 0.0
+    tol = 8 * max(nb, 1) * 2.0 ** -24 if single else 1e-10
+    res["ok"] = res["info_oracle"] == res["info_gpu"] and res["bwd"] <= 10.0 and res["rowscaled"] <= tol
+    return res

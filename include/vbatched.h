@@ -187,6 +187,25 @@ int vbatched_dposv(char uplo, const int* d_n, const int* d_nrhs, double* const* 
                    int batchCount, int max_n, int max_nrhs, vb_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------
+ * vbatched_zpotrf / vbatched_cpotrf — variable-size batched complex Cholesky A_i = L_i L_i^H
+ * (uplo 'L') or U_i^H U_i (uplo 'U') of Hermitian positive definite matrices (SURVEY.md §8(f)
+ * NEXT-3; the paper's framework "supports complex precisions", §IV-A;
+ * LAPACK ZPOTRF / CPOTRF semantics).
+ *  dA_array   [batchCount] device pointers to complex matrices, interleaved (re, im) per element,
+ *             column-major: element (r,c) of matrix i is ((T*)dA_array[i])[2*(r + c*ldda[i])]
+ *             (+1 for the imaginary part); T = double (Z) or float (C). Only the `uplo`
+ *             triangle is referenced; the diagonal's imaginary part is ignored on input and
+ *             written as 0 in the factor. 16-byte (Z) / 8-byte (C) aligned.
+ *  Everything else (d_n, d_ldda in elements, d_info codes incl. -2/-4/-7 and k > 0, max_n,
+ *  return codes) exactly as vbatched_dpotrf. CPOTRF stores FP32 and computes in FP64 (as
+ *  vbatched_spotrf). Complex products on the FP64 tensor cores are four real DMMAs.
+ */
+int vbatched_zpotrf(char uplo, const int* d_n, void* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream);
+int vbatched_cpotrf(char uplo, const int* d_n, void* const* dA_array, const int* d_ldda,
+                    int* d_info, int batchCount, int max_n, vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
  * vbatched_dgetrf — FP64 variable-size batched LU with partial pivoting, A_i = P_i L_i U_i
  * (the LU extension the paper names as future work, PAPER.md:2279-2285
  * §V, built from its vbatched kernels, §III-E; LAPACK DGETRF semantics).

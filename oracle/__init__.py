@@ -64,6 +64,13 @@ def lib():
         L.oracle_getrf_backward_error.argtypes = [ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int, _dp,
                                                   ctypes.c_int, _ip]
         L.oracle_getrf_backward_error.restype = ctypes.c_double
+        L.oracle_zpotrf_lower.argtypes = [ctypes.c_int, _dp, ctypes.c_int]
+        L.oracle_zpotrf_lower.restype = ctypes.c_int
+        L.oracle_cpotrf_lower.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_float), ctypes.c_int]
+        L.oracle_cpotrf_lower.restype = ctypes.c_int
+        L.oracle_zpotrf_backward_error.argtypes = [ctypes.c_int, _dp, ctypes.c_int, _dp, ctypes.c_int,
+                                                   ctypes.c_int]
+        L.oracle_zpotrf_backward_error.restype = ctypes.c_double
         L.oracle_backward_error_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip,
                                                   ctypes.POINTER(_dp), _ip, _ip, _dp, ctypes.c_int]
         _lib = L
@@ -230,3 +237,30 @@ def getrf_backward_error(A0: np.ndarray, F: np.ndarray, ipiv: np.ndarray) -> flo
         ip = np.zeros(1, np.int32)
     return lib().oracle_getrf_backward_error(m, n, _ptr(A0), max(1, m), _ptr(F), max(1, F.shape[0]),
                                              ip.ctypes.data_as(_ip))
+
+
+def zpotrf(a: np.ndarray) -> tuple[np.ndarray, int]:
+    """Oracle complex Cholesky A = L L^H of one Hermitian matrix (complex128; only its lower
+    triangle is read, the diagonal's imaginary part ignored). Returns (copy with L in the lower
+    triangle, info)."""
+    out = np.array(a, dtype=np.complex128, order="F", copy=True)
+    n = out.shape[0]
+    info = lib().oracle_zpotrf_lower(n, out.ctypes.data_as(_dp), max(1, n))
+    return out, info
+
+
+def cpotrf(a: np.ndarray) -> tuple[np.ndarray, int]:
+    """The same recurrence in IEEE single precision (complex64)."""
+    out = np.array(a, dtype=np.complex64, order="F", copy=True)
+    n = out.shape[0]
+    info = lib().oracle_cpotrf_lower(n, out.ctypes.data_as(ctypes.POINTER(ctypes.c_float)), max(1, n))
+    return out, info
+
+
+def zpotrf_backward_error(A0: np.ndarray, L: np.ndarray, info: int) -> float:
+    """||A - L L^H||_F / (nb ||A||_F 2^-53), long double (complex; SURVEY §8(c) #13 extended)."""
+    A0 = np.asfortranarray(A0, dtype=np.complex128)
+    L = np.asfortranarray(L, dtype=np.complex128)
+    n = A0.shape[0]
+    return lib().oracle_zpotrf_backward_error(n, A0.ctypes.data_as(_dp), max(1, n), L.ctypes.data_as(_dp),
+                                              max(1, L.shape[0]), int(info))

@@ -36,6 +36,14 @@
  *    (IEEE division), rank-1 update a_ij -= l_ik u_kj in k order; a zero pivot records
  *    info = k+1 (first only) and elimination continues (nothing to scale: the column is zero).
  *  - oracle_getrf_backward_error: ||P A - L U||_F / (max(m,n) ||A||_F eps), long double.
+ *  - oracle_zpotrf_lower / oracle_cpotrf_lower: the complex Hermitian problem A = L L^H (the
+ *    paper's "supports complex precisions", §IV-A; LAPACK ZPOTRF/CPOTRF;
+ *    SURVEY.md §8(f) NEXT-3). The same Crout recurrence with conjugates,
+ *        l_jj = sqrt(Re a_jj - sum_{k<j} |l_jk|^2),  l_ij = (a_ij - sum_{k<j} l_ik conj(l_jk)) / l_jj,
+ *    complex arithmetic written out in real operations (no C99 complex), k ascending; the
+ *    imaginary part of the diagonal is ignored and stored as 0 (LAPACK). Interleaved storage
+ *    (re, im) per element, column-major. Double (Z) and single (C) precision.
+ *  - oracle_zpotrf_backward_error: ||A - L L^H||_F / (n ||A||_F eps), long double, eps = 2^-53.
  */
 #include <math.h>
 #include <stdlib.h>
@@ -351,4 +359,88 @@ double oracle_getrf_backward_error(int m, int n, const double* A0, int lda0, con
   const long double eps = ldexpl(1.0L, -53);
   const int mx = m > n ? m : n;
   return (double)(sqrtl(num) / ((long double)mx * sqrtl(den) * eps));
+}
+
+/* Complex Cholesky-Crout on the lower triangle of an interleaved column-major n x n Hermitian
+ * matrix (element (i,j) at a[2*(i + j*lda)] (re), [.. + 1] (im)). Returns LAPACK info. */
+#define ZPOTRF_BODY(T, SQRT)                                                                    \
+  if (n <= 0) return 0;                                                                        \
+  T* w = (T*)malloc(sizeof(T) * 2 * (size_t)n * (size_t)n); /* row-major lower: w[2*(i*n+j)] */ \
+  if (!w) return -1000;                                                                        \
+  for (int i = 0; i < n; ++i)                                                                  \
+    for (int j = 0; j <= i; ++j) {                                                             \
+      w[2 * ((size_t)i * n + j)] = a[2 * IDX(i, j, lda)];                                      \
+      w[2 * ((size_t)i * n + j) + 1] = (i == j) ? (T)0 : a[2 * IDX(i, j, lda) + 1];            \
+    }                                                                                          \
+  int info = 0, done = n;                                                                      \
+  for (int j = 0; j < n; ++j) {                                                                \
+    const T* lj = w + 2 * (size_t)j * n;                                                       \
+    T s = lj[2 * j];                                                                           \
+    for (int k = 0; k < j; ++k) s = s - (lj[2 * k] * lj[2 * k] + lj[2 * k + 1] * lj[2 * k + 1]); \
+    if (!(s > (T)0)) {                                                                         \
+      w[2 * ((size_t)j * n + j)] = s;                                                          \
+      info = j + 1;                                                                            \
+      done = j;                                                                                \
+      break;                                                                                   \
+    }                                                                                          \
+    const T ljj = SQRT(s);                                                                     \
+    w[2 * ((size_t)j * n + j)] = ljj;                                                          \
+    w[2 * ((size_t)j * n + j) + 1] = (T)0;                                                     \
+    for (int i = j + 1; i < n; ++i) {                                                          \
+      T* li = w + 2 * (size_t)i * n;                                                           \
+      T tr = li[2 * j], ti = li[2 * j + 1];                                                    \
+      for (int k = 0; k < j; ++k) {                                                            \
+        /* l_ik conj(l_jk) = (ar + i ai)(br - i bi) = (ar br + ai bi) + i (ai br - ar bi) */  \
+        const T ar = li[2 * k], ai = li[2 * k + 1], br = lj[2 * k], bi = lj[2 * k + 1];        \
+        tr = tr - (ar * br + ai * bi);                                                         \
+        ti = ti - (ai * br - ar * bi);                                                         \
+      }                                                                                        \
+      li[2 * j] = tr / ljj;                                                                    \
+      li[2 * j + 1] = ti / ljj;                                                                \
+    }                                                                                          \
+  }                                                                                            \
+  for (int j = 0; j < done; ++j)                                                               \
+    for (int i = j; i < n; ++i) {                                                              \
+      a[2 * IDX(i, j, lda)] = w[2 * ((size_t)i * n + j)];                                      \
+      a[2 * IDX(i, j, lda) + 1] = w[2 * ((size_t)i * n + j) + 1];                              \
+    }                                                                                          \
+  if (info > 0) {                                                                              \
+    a[2 * IDX(info - 1, info - 1, lda)] = w[2 * ((size_t)(info - 1) * n + (info - 1))];        \
+    a[2 * IDX(info - 1, info - 1, lda) + 1] = (T)0;                                            \
+  }                                                                                            \
+  free(w);                                                                                     \
+  return info;
+
+int oracle_zpotrf_lower(int n, double* a, int lda) { ZPOTRF_BODY(double, sqrt) }
+int oracle_cpotrf_lower(int n, float* a, int lda) { ZPOTRF_BODY(float, sqrtf) }
+
+/* ||A - L L^H||_F / (nb ||A||_F eps), eps = 2^-53, long double; A Hermitian rebuilt from the
+ * lower triangle of A0 (diagonal imaginary part ignored), L = lower triangle of Lf (upper taken
+ * as zero, diagonal imaginary part as stored). nb = n, or info-1 on failure. */
+double oracle_zpotrf_backward_error(int n, const double* A0, int lda0, const double* Lf, int ldl,
+                                    int info) {
+  int nb = info > 0 ? info - 1 : n;
+  if (nb <= 0) return 0.0;
+  long double num = 0.0L, den = 0.0L;
+  for (int j = 0; j < nb; ++j)
+    for (int i = 0; i < nb; ++i) {
+      long double ar, ai;
+      if (i > j) { ar = A0[2 * IDX(i, j, lda0)]; ai = A0[2 * IDX(i, j, lda0) + 1]; }
+      else if (i < j) { ar = A0[2 * IDX(j, i, lda0)]; ai = -(long double)A0[2 * IDX(j, i, lda0) + 1]; }
+      else { ar = A0[2 * IDX(i, i, lda0)]; ai = 0.0L; }
+      long double sr = 0.0L, si = 0.0L;
+      const int kmax = i < j ? i : j;
+      for (int k = 0; k <= kmax; ++k) {
+        const long double xr = Lf[2 * IDX(i, k, ldl)], xi = Lf[2 * IDX(i, k, ldl) + 1];
+        const long double yr = Lf[2 * IDX(j, k, ldl)], yi = Lf[2 * IDX(j, k, ldl) + 1];
+        sr += xr * yr + xi * yi;
+        si += xi * yr - xr * yi;
+      }
+      const long double dr = ar - sr, di = ai - si;
+      num += dr * dr + di * di;
+      den += ar * ar + ai * ai;
+    }
+  if (den == 0.0L) return num == 0.0L ? 0.0 : INFINITY;
+  const long double eps = ldexpl(1.0L, -53);
+  return (double)(sqrtl(num) / ((long double)nb * sqrtl(den) * eps));
 }

@@ -20,7 +20,7 @@ __all__ = [
     "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
     "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "vbatched_dpotrf_kernel_names",
-    "vbatched_release_host_staging", "factor_kernel_names", "vbatched_dgetrf", "lib", "LIB_PATH", "VBatchedError",
+    "vbatched_release_host_staging", "factor_kernel_names", "vbatched_dgetrf", "vbatched_zpotrf", "vbatched_cpotrf", "lib", "LIB_PATH", "VBatchedError",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -68,6 +68,8 @@ def lib() -> ctypes.CDLL:
         L.vbatched_dpotrf_kernel_launches.restype = _i
         L.vbatched_dpotrf_kernel_names.argtypes = [_i]
         L.vbatched_dpotrf_kernel_names.restype = ctypes.c_char_p
+        L.vbatched_zpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
+        L.vbatched_cpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
         L.vbatched_dgetrf.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_release_host_staging.argtypes = []
         L.vbatched_release_host_staging.restype = _i
@@ -208,6 +210,21 @@ def vbatched_dposv(uplo, n, nrhs, dA_array, ldda, dB_array, lddb, info, batchCou
                               _ptr(dB_array), _ptr(lddb), _ptr(info), int(batchCount), int(max_n),
                               int(max_nrhs), _stream(stream))
     return _check(rc, "vbatched_dposv") if check else rc
+
+
+def vbatched_zpotrf(uplo, n, dA_array, ldda, info, batchCount, max_n, stream=None, check=True):
+    """vbatched complex<double> Cholesky (include/vbatched.h): matrices as complex128 tensors'
+    addresses in dA_array (int64 device pointers)."""
+    rc = lib().vbatched_zpotrf(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
+                               int(batchCount), int(max_n), _stream(stream))
+    return _check(rc, "vbatched_zpotrf") if check else rc
+
+
+def vbatched_cpotrf(uplo, n, dA_array, ldda, info, batchCount, max_n, stream=None, check=True):
+    """vbatched complex<float> Cholesky (FP32 storage, FP64 arithmetic)."""
+    rc = lib().vbatched_cpotrf(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
+                               int(batchCount), int(max_n), _stream(stream))
+    return _check(rc, "vbatched_cpotrf") if check else rc
 
 
 def vbatched_dgetrf(m, n, dA_array, ldda, dipiv_array, info, batchCount, max_m, max_n, stream=None,

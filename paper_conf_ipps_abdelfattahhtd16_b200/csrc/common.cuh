@@ -168,6 +168,14 @@ VB_DEVINL void fence_proxy_async_global() {
 VB_DEVINL void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
 VB_DEVINL void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;\n" ::); }
 
+// Named barriers (bar.sync / bar.arrive on a subset of the CTA's warps).
+VB_DEVINL void bar_group(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
+}
+VB_DEVINL void bar_group_arrive(int id, int nthreads) {
+  asm volatile("bar.arrive %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
+}
+
 constexpr int LDS_T = 18;  // TRTRI32 scratch leading dim (16 columns used)
 
 // Inverse of a 32x32 lower-triangular L (T[c*ldt+r] = L[r][c], tv[c] = 1/L[c][c]) by one

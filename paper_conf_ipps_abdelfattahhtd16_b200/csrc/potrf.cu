@@ -281,12 +281,6 @@ VB_DEVINL void mm32_quarter(double (&acc)[2][2][2], int wg, int lane, FA fa, FB 
   }
 }
 
-VB_DEVINL void bar_group(int id, int nthreads) {
-  asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
-}
-VB_DEVINL void bar_group_arrive(int id, int nthreads) {
-  asm volatile("bar.arrive %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
-}
 
 // =======================================================================================
 // Blocked kernel (n > ts) building blocks: warp w owns 16 full rows of each MB-row block, so

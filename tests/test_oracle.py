@@ -693,3 +693,72 @@ def test_lu_backward_error_gate_closed_form():
     G = vbgen.g1_matrix(2, 9, 200, 200)
     FG, ipg, _ = oracle.dgetrf(G)
     assert oracle.getrf_backward_error(G, FG, ipg) < 10
+
+
+# ---------------------------------------------------------------- complex Cholesky (NEXT-3)
+def test_zpotrf_handworked():
+    """[[4, .], [2+2i, 6]] -> l21 = 1+i, l22 = sqrt(6 - |1+i|^2) = 2 (exact); the strict upper
+    triangle is never read or written; the diagonal's imaginary part is ignored."""
+    A = np.array([[4 + 5j, np.nan], [2 + 2j, 6 - 3j]], dtype=np.complex128)
+    L, info = oracle.zpotrf(A)
+    assert info == 0
+    assert L[0, 0] == 2 and L[1, 0] == 1 + 1j and L[1, 1] == 2
+    assert np.isnan(L[0, 1])
+
+
+@pytest.mark.parametrize("n", [1, 7, 33, 100])
+def test_zpotrf_gaussian_integer_family_exact(n):
+    """L with real diagonal in {1,2,4} and Gaussian-integer entries in {-1,0,1} + i{-1,0,1}:
+    A = L L^H is exact, so chol(A) = L bit for bit (double and single precision)."""
+    rng = np.random.default_rng(300 + n)
+    L = np.tril(rng.integers(-1, 2, (n, n)) + 1j * rng.integers(-1, 2, (n, n)), -1)
+    L[np.arange(n), np.arange(n)] = rng.choice([1.0, 2.0, 4.0], n)
+    A = L @ L.conj().T
+    Lz, info = oracle.zpotrf(A)
+    assert info == 0 and np.array_equal(np.tril(Lz), L)
+    if n <= 33:
+        Lc, info = oracle.cpotrf(A.astype(np.complex64))
+        assert info == 0 and np.array_equal(np.tril(Lc), L.astype(np.complex64))
+
+
+def test_zpotrf_real_case_equals_real_oracle():
+    """With zero imaginary parts the complex recurrence performs the real one's operations."""
+    A = vbgen.f1_matrix(3, 4, 60)
+    Lr, ir = oracle.dpotrf(A)
+    Lz, iz = oracle.zpotrf(A.astype(np.complex128))
+    assert ir == iz == 0
+    assert np.array_equal(np.tril(Lz).real, np.tril(Lr)) and not np.tril(Lz).imag.any()
+
+
+@pytest.mark.parametrize("n", [5, 64, 200])
+def test_zpotrf_matches_lapack_and_backward_error(n):
+    import torch
+    A = vbgen.f1c_matrix(9, n, n)
+    L, info = oracle.zpotrf(A)
+    assert info == 0
+    ref = np.linalg.cholesky(A)  # LAPACK ZPOTRF (numpy's bundled OpenBLAS)
+    assert np.max(np.abs(np.tril(L) - ref)) <= 1e-13 * np.max(np.abs(ref))
+    Lt, it = torch.linalg.cholesky_ex(torch.from_numpy(A))  # MKL
+    assert int(it) == 0 and np.max(np.abs(np.tril(L) - Lt.numpy())) <= 1e-13 * np.max(np.abs(ref))
+    assert oracle.zpotrf_backward_error(A, np.tril(L), 0) < 10
+    Lc, infoc = oracle.cpotrf(A.astype(np.complex64))
+    assert infoc == 0 and np.max(np.abs(np.tril(Lc) - ref)) <= 8 * n * 2.0 ** -24 * np.max(np.abs(ref))
+
+
+def test_zpotrf_info_and_backward_error_gate():
+    A = vbgen.f1c_matrix(4, 19, 40, nonspd=True)
+    k = vbgen.nonspd_k(4, 19, 40)
+    L, info = oracle.zpotrf(A)
+    assert info == k
+    # closed-form gate: a perturbation d of one entry of an exact factor
+    rng = np.random.default_rng(2)
+    n = 5
+    Le = np.tril(rng.integers(-1, 2, (n, n)) + 1j * rng.integers(-1, 2, (n, n)), -1)
+    Le[np.arange(n), np.arange(n)] = 2.0
+    Ae = Le @ Le.conj().T
+    assert oracle.zpotrf_backward_error(Ae, Le, 0) == 0.0
+    Lp = Le.copy()
+    Lp[3, 1] += 2.0 ** -40 * 1j
+    D = Ae - Lp @ Lp.conj().T  # exact in double: entries are Gaussian integers +- 2^-40 terms
+    exp = np.sqrt(np.sum(np.abs(D) ** 2)) / (n * np.sqrt(np.sum(np.abs(Ae) ** 2)) * 2.0 ** -53)
+    assert oracle.zpotrf_backward_error(Ae, Lp, 0) == pytest.approx(exp, rel=1e-9)

@@ -139,6 +139,30 @@ def g1_matrix(seed: int, gidx: int, m: int, n: int) -> np.ndarray:
     return np.asfortranarray(2.0 * u - 1.0)
 
 
+def f1c_matrix(seed: int, gidx: int, n: int, nonspd: bool = False) -> np.ndarray:
+    """Complex Hermitian family F1c (complex Cholesky): a_ij = u + i v
+    (i > j, u, v from the counter hash keyed by (gidx, i, j) and (gidx, i, j) ^ 2^62), a_ji =
+    conj(a_ij), a_ii = u_ii + 2n (real): diagonally dominant (|a_ij| < sqrt 2), so Hermitian PD.
+    nonspd negates a_kk at the same hashed k as F1. Input generation only."""
+    if n == 0:
+        return np.zeros((0, 0), dtype=np.complex128, order="F")
+    i = np.arange(n)[:, None] + np.zeros((1, n), np.int64)
+    j = np.arange(n)[None, :] + np.zeros((n, 1), np.int64)
+    hi, lo = np.maximum(i, j), np.minimum(i, j)
+    re = _u(seed, gidx, hi, lo)
+    key = (np.uint64(gidx) << np.uint64(42)) ^ (hi.astype(np.uint64) << np.uint64(21)) ^ \
+        lo.astype(np.uint64) ^ np.uint64(1 << 62)
+    im = (splitmix64(splitmix64(np.uint64(seed)) ^ key) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+    im = np.where(i > j, im, -im)
+    a = re + 1j * im
+    d = np.arange(n)
+    a[d, d] = re[d, d] + 2.0 * n
+    if nonspd:
+        k = nonspd_k(seed, gidx, n) - 1
+        a[k, k] = -a[k, k]
+    return np.asfortranarray(a)
+
+
 def config_matrix(cfg: Config | str, gidx: int, n: int | None = None) -> np.ndarray:
     if isinstance(cfg, str):
         cfg = CONFIGS[cfg]
