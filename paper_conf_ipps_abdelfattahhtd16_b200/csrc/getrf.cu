@@ -21,7 +21,7 @@
 namespace vb {
 namespace {
 
-constexpr int kLuNB = 16;        // panel width
+constexpr int kLuNB = 16;        // panel width (the trailing GEMM's k)
 constexpr int kLuThreads = 256;  // panel kernel CTA
 constexpr int kLuMaxRPT = 4;     // rows per thread held in registers: m - j <= 1024
 
@@ -194,28 +194,65 @@ __global__ void __launch_bounds__(kLuThreads)
 }
 
 // Row interchanges of the step's pivots on the columns outside the panel (LAPACK DLASWP on
-// columns 0..j-1 and j+pn..n-1): one CTA per matrix, a thread per column, pivots in order.
+// columns 0..j-1 and j+pn..n-1). The pn sequential swaps only move rows of the set
+// S = {j..j+pn-1} u {ipiv targets} (<= 2 pn <= 64 rows); their composition is a permutation pi
+// of S, built once per matrix in shared memory. Then one warp per column: each lane loads two
+// rows of S (one coalesced run j..j+pn-1, the rest scattered), and writes row S[t] with the
+// value of row pi(S[t]) taken by a shuffle — one gather and one scatter per column instead of
+// 2 pn dependent strided accesses.
 __global__ void __launch_bounds__(256)
     lu_laswp_kernel(LuStep st, double* const* __restrict__ dA, const int* __restrict__ d_n,
                     const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv, int batch, int j) {
+  __shared__ int srow[2 * kLuNB];  // S
+  __shared__ int ssrc[2 * kLuNB];  // for slot t: the slot whose old value moves to S[t]
+  __shared__ int s_cnt;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   for (int i = blockIdx.x; i < batch; i += gridDim.x) {
     const int pn = st.pn[i];
     if (pn <= 0) continue;
     const int n = d_n[i], ld = d_ld[i];
     double* A = dA[i];
     const int* ip = d_ipiv[i] + j;
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
+    if (threadIdx.x == 0) {
+      // slots 0..pn-1: rows j..j+pn-1; further slots: targets outside that range
+      int cnt = pn;
+      int cur[2 * kLuNB];  // cur[t]: slot whose original value currently sits in S[t]
+      for (int t = 0; t < pn; ++t) {
+        srow[t] = j + t;
+        cur[t] = t;
+      }
+      for (int k = 0; k < pn; ++k) {
+        const int r2 = ip[k] - 1;
+        int t2 = -1;
+        for (int t = 0; t < cnt; ++t)
+          if (srow[t] == r2) t2 = t;
+        if (t2 < 0) {
+          t2 = cnt++;
+          srow[t2] = r2;
+          cur[t2] = t2;
+        }
+        const int x = cur[k];
+        cur[k] = cur[t2];
+        cur[t2] = x;
+      }
+      for (int t = 0; t < cnt; ++t) ssrc[t] = cur[t];
+      s_cnt = cnt;
+    }
+    __syncthreads();
+    const int cnt = s_cnt;
+    const int r_lo = lane < cnt ? srow[lane] : 0, r_hi = lane + 32 < cnt ? srow[lane + 32] : 0;
+    const int f_lo = lane < cnt ? ssrc[lane] : 0, f_hi = lane + 32 < cnt ? ssrc[lane + 32] : 0;
+    for (int c = warp; c < n; c += nw) {
       if (c >= j && c < j + pn) continue;
       double* col = A + (size_t)c * ld;
-      for (int k = 0; k < pn; ++k) {
-        const int r2 = ip[k] - 1, r1 = j + k;
-        if (r2 != r1) {
-          const double t = col[r1];
-          col[r1] = col[r2];
-          col[r2] = t;
-        }
-      }
+      const double v_lo = lane < cnt ? col[r_lo] : 0.0;
+      const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
+      const double a_lo = __shfl_sync(kFull, v_lo, f_lo & 31), b_lo = __shfl_sync(kFull, v_hi, f_lo & 31);
+      const double a_hi = __shfl_sync(kFull, v_lo, f_hi & 31), b_hi = __shfl_sync(kFull, v_hi, f_hi & 31);
+      if (lane < cnt) col[r_lo] = f_lo < 32 ? a_lo : b_lo;
+      if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
     }
+    __syncthreads();
   }
 }
 
