@@ -88,6 +88,11 @@ VB_DEVINL void cp_async16(void* sdst, const void* gsrc, bool pred) {
 VB_DEVINL void cp_async_mbar_arrive(uint64_t* bar) {
   asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
+// The barrier receives this thread's arrival once all its prior cp.async copies have completed
+// (the pending count is not incremented: the arrival counts toward the phase's expected count).
+VB_DEVINL void cp_async_mbar_arrive_noinc(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
 VB_DEVINL void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 template <int N>
 VB_DEVINL void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }

@@ -415,9 +415,12 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
     // G here) and only ever feed output rows/columns that are never stored
     const int ra = (min(C::MB, n - r0) + G - 1) / G * G;
     const int rb = (min(C::NB, n - j0) + G - 1) / G * G;
+    // the full barrier expects one arrival per producer lane (see the gather path below): lane
+    // 0 arrives with the transaction count, the others plainly
     if (lane == 0)
       mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * (int)sizeof(E)));
     __syncwarp();
+    if (lane != 0) mbar_arrive(&s.full[st]);
     if (lane < C::KC) {
       // A rows stream (re-read only a panel later): evict first; the panel rows are re-read
       // for every row block of the panel: evict last (C5 DRAM traffic and time)
@@ -432,8 +435,8 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
     // Odd ldda / unaligned base ('L'), or uplo 'U': the chunk is gathered with 8-byte cp.async
     // (LDGSTS, no register staging; rows >= n are zero-filled). 'L': lanes run down a column;
     // 'U': L's rows are contiguous in storage (16 k-values of one row = 128 B), 16 lanes per
-    // row. Every lane's copies are tracked by the full barrier (cp.async.mbarrier.arrive: zero
-    // net arrivals) and lane 0 adds the one expected arrival.
+    // row. Each lane's arrival on the full barrier is its cp.async.mbarrier.arrive.noinc,
+    // triggered when all of that lane's copies have landed (32 expected arrivals per phase).
     static_assert(C::KC == 16 && C::MB % 32 == 0 && C::NB % 32 == 0, "copy shapes");
     if (UP) {
       const int c = lane & 15;
@@ -463,9 +466,7 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
         }
       }
     }
-    cp_async_mbar_arrive(&s.full[st]);
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&s.full[st]);
+    cp_async_mbar_arrive_noinc(&s.full[st]);
   }
 }
 
@@ -764,7 +765,7 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
   if (threadIdx.x == 0) {
     for (int i = 0; i < C::STAGES; ++i) {
-      mbar_init(&s.full[i], 1);
+      mbar_init(&s.full[i], 32);  // one arrival per producer lane
       mbar_init(&s.empty[i], kV3Consumers);
     }
     mbar_init(&s.panel_done, kV3Consumers);

@@ -42,7 +42,8 @@ struct ZSmem {
   double2 inv[kZNB][kZLD];  // inv[k][c] = Linv(c, k): the TRSM's B operand (conjugated there)
   double2 col[kZNB];        // POTF2 column broadcast
   int item;
-  int info;
+  int info[2];  // panel p's pivot status in info[p & 1]: read by every warp at the end of panel
+                // p while warp 0 may already write panel p+1's
 };
 
 // L(r, c) (r >= c) of matrix storage A with uplo: 'L' keeps L, 'U' keeps U = L^H, so L(r, c) =
@@ -155,6 +156,7 @@ VB_DEVINL int zpotf2_warp(ZSmem& s, int nb, E2* __restrict__ Ad, int ld, int lan
   double2 a[kZNB];
 #pragma unroll
   for (int c = 0; c < kZNB; ++c) a[c] = (c <= r && r < nb) ? s.T[c][r] : make_double2(0.0, 0.0);
+  __syncwarp();  // lanes 16..31 mirror rows 0..15: their reads precede lanes 0..15's writes below
   int info = 0, ncol = nb;
 #pragma unroll
   for (int j = 0; j < kZNB; ++j) {
@@ -246,7 +248,7 @@ VB_DEVINL void zpotrf_matrix(ZSmem& s, E2* __restrict__ A, int n, int ld, int* i
       const int info = zpotf2_warp<UP, E2>(s, nb, A + (size_t)j0 * ld + j0, ld, lane);
       if (!info && below) ztrtri_warp(s, nb, lane);
       if (lane == 0) {
-        s.info = info;
+        s.info[p & 1] = info;
         if (info) *info_out = j0 + info;
       }
       if (below) bar_group_arrive(1, 128);
@@ -261,13 +263,13 @@ VB_DEVINL void zpotrf_matrix(ZSmem& s, E2* __restrict__ A, int n, int ld, int* i
           bar_group(1, 128);
           synced = true;
         }
-        if (s.info) break;
+        if (s.info[p & 1]) break;
         zstrip_trsm_store<UP, E2>(s, ar, ai, A, n, ld, r0, j0, lane);
       }
       if (!synced) bar_group(1, 128);
     }
-    __syncthreads();  // the panel's L is stored before the next panel reads it; s.info settled
-    if (s.info) return;
+    __syncthreads();  // the panel's L is stored before the next panel reads it; info settled
+    if (s.info[p & 1]) return;
   }
 }
 
@@ -283,10 +285,7 @@ __global__ void __launch_bounds__(128, 4)
                     *(volatile const int*)&ctrl->count[2];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   for (;;) {
-    if (threadIdx.x == 0) {
-      s.item = atomicAdd(&ctrl->head[0], 1);
-      s.info = 0;
-    }
+    if (threadIdx.x == 0) s.item = atomicAdd(&ctrl->head[0], 1);
     __syncthreads();
     const int it = s.item;
     __syncthreads();

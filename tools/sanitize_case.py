@@ -5,6 +5,8 @@ overhead, covering every kernel and protocol of one vbatched_dpotrf call (VERDIC
   mixed  200 matrices spanning all three factorisation kernels (n in 1..700), 'L' and 'U',
          roundup-32 and odd ldda (the cp.async gather instead of TMA bulk copies), failing
          pivots (-> early termination, the TMA ring drain, the look-ahead barrier exits).
+  lu     vbatched_dgetrf on 40 general matrices (square and rectangular, n < 300).
+  z      vbatched_zpotrf / vbatched_cpotrf with non-HPD matrices.
 Each case checks info against the expected values so a silent corruption also fails.
 """
 import os
@@ -26,9 +28,10 @@ def c1():
     assert np.all(db.info() == 0)
 
 
-def mixed():
+def mixed(scale=1):
     rng = np.random.default_rng(200)
-    n = np.concatenate([rng.integers(1, 33, 60), rng.integers(33, 129, 80), rng.integers(129, 701, 60)]).astype(np.int32)
+    n = np.concatenate([rng.integers(1, 33, 60 // scale), rng.integers(33, 129, 80 // scale),
+                        rng.integers(129, 701, 60 // scale)]).astype(np.int32)
     for uplo in ("L", "U"):
         for mode in ("pad32", "odd"):
             db = DeviceBatch(n, seed=201, nonspd_mod=9, ldda_mode=mode).fill(poison=True, uplo=uplo)
@@ -40,6 +43,29 @@ def mixed():
     print("mixed ok")
 
 
+def lu():
+    from harness import LUBatch
+    rng = np.random.default_rng(7)
+    n = rng.integers(1, 300, 40).astype(np.int32)
+    m = n.copy()
+    m[::5] = np.maximum(1, n[::5] // 2)
+    lb = LUBatch(m, n, seed=3).fill()
+    lb.getrf()
+    torch.cuda.synchronize()
+    assert np.all(lb.info() == 0)
+
+
+def z():
+    from harness import ZBatch
+    n = np.array([1, 5, 16, 17, 40, 100, 200], np.int32)
+    for single in (False, True):
+        zb = ZBatch(n, seed=5, single=single, nonspd_mod=3).fill()
+        zb.potrf()
+        torch.cuda.synchronize()
+        exp = [vbgen.nonspd_k(5, i, int(n[i])) if i % 3 == 2 else 0 for i in range(len(n))]
+        assert list(zb.info()) == exp
+
+
 if __name__ == "__main__":
-    {"c1": c1, "mixed": mixed}[sys.argv[1]]()
+    {"c1": c1, "mixed": mixed, "mixed_small": lambda: mixed(4), "lu": lu, "z": z}[sys.argv[1]]()
     print("case ok", sys.argv[1])
