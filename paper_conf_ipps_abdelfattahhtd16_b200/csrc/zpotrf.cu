@@ -70,7 +70,8 @@ VB_DEVINL void zstrip_kloop(double (&ar)[2][2][2], double (&ai)[2][2][2], const 
   const int g = lane >> 2, q = lane & 3;
   const bool rv0 = r0 + g < n, rv1 = r0 + 8 + g < n, cv0 = c0 + g < n, cv1 = c0 + 8 + g < n;
 #pragma unroll 2
-  for (int k = kb + q; k < ke; k += 4) {
+  for (int k0 = kb; k0 < ke; k0 += 4) {  // warp-uniform trip count (mma.sync.aligned)
+    const int k = k0 + q;
     double2 a0 = rv0 ? ld_l<UP>(A, r0 + g, k, ld) : make_double2(0.0, 0.0);
     double2 a1 = rv1 ? ld_l<UP>(A, r0 + 8 + g, k, ld) : make_double2(0.0, 0.0);
     double2 b0 = cv0 ? ld_l<UP>(A, c0 + g, k, ld) : make_double2(0.0, 0.0);
