@@ -71,6 +71,11 @@ def lib():
         L.oracle_zpotrf_backward_error.argtypes = [ctypes.c_int, _dp, ctypes.c_int, _dp, ctypes.c_int,
                                                    ctypes.c_int]
         L.oracle_zpotrf_backward_error.restype = ctypes.c_double
+        L.oracle_dgeqrf.argtypes = [ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int, _dp]
+        L.oracle_dgeqrf.restype = None
+        L.oracle_geqrf_errors.argtypes = [ctypes.c_int, ctypes.c_int, _dp, ctypes.c_int, _dp, ctypes.c_int,
+                                          _dp, _dp, _dp]
+        L.oracle_geqrf_errors.restype = None
         L.oracle_backward_error_batch.argtypes = [ctypes.c_int, _ip, ctypes.POINTER(_dp), _ip,
                                                   ctypes.POINTER(_dp), _ip, _ip, _dp, ctypes.c_int]
         _lib = L
@@ -264,3 +269,27 @@ def zpotrf_backward_error(A0: np.ndarray, L: np.ndarray, info: int) -> float:
     n = A0.shape[0]
     return lib().oracle_zpotrf_backward_error(n, A0.ctypes.data_as(_dp), max(1, n), L.ctypes.data_as(_dp),
                                               max(1, L.shape[0]), int(info))
+
+
+def dgeqrf(a: np.ndarray) -> tuple[np.ndarray, np.ndarray]:
+    """Oracle Householder QR (oracle.c: textbook DGEQR2 / DLARFG conventions). Returns (compact
+    factor: R on/above the diagonal, v below; tau[min(m,n)])."""
+    out = np.array(a, dtype=np.float64, order="F", copy=True)
+    m, n = out.shape
+    tau = np.zeros(max(1, min(m, n)))
+    lib().oracle_dgeqrf(m, n, _ptr(out), max(1, m), _ptr(tau))
+    return out, tau[: min(m, n)]
+
+
+def geqrf_errors(A0: np.ndarray, F: np.ndarray, tau: np.ndarray) -> tuple[float, float]:
+    """(||A - QR||_F / (max(m,n) ||A||_F eps), ||Q^T Q - I||_F / (m eps)), long double."""
+    A0 = np.asfortranarray(A0, dtype=np.float64)
+    F = np.asfortranarray(F, dtype=np.float64)
+    m, n = A0.shape
+    t = np.ascontiguousarray(tau, dtype=np.float64)
+    if t.size == 0:
+        t = np.zeros(1)
+    b, o = ctypes.c_double(), ctypes.c_double()
+    lib().oracle_geqrf_errors(m, n, _ptr(A0), max(1, m), _ptr(F), max(1, F.shape[0]), _ptr(t),
+                              ctypes.byref(b), ctypes.byref(o))
+    return b.value, o.value

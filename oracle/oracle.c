@@ -44,6 +44,13 @@
  *    imaginary part of the diagonal is ignored and stored as 0 (LAPACK). Interleaved storage
  *    (re, im) per element, column-major. Double (Z) and single (C) precision.
  *  - oracle_zpotrf_backward_error: ||A - L L^H||_F / (n ||A||_F eps), long double, eps = 2^-53.
+ *  - oracle_dgeqrf: Householder QR, A = Q R (the QR extension named as future work,
+ *    PAPER.md:2279-2285, §V), textbook unblocked form with LAPACK
+ *    DGEQR2 / DLARFG conventions: for column k, alpha = a_kk, xnorm = ||a_(k+1:m, k)||_2 (plain
+ *    sum of squares, k ascending), beta = -sign(alpha) sqrt(alpha^2 + xnorm^2), tau = (beta -
+ *    alpha) / beta, v = a_(k+1:m, k) / (alpha - beta) (IEEE division), a_kk = beta; then
+ *    H_k = I - tau v v^T (v_0 = 1) applied to columns k+1..n-1: w = v^T a_j, a_j -= tau w v.
+ *    xnorm == 0 gives tau = 0 (H = I). R on and above the diagonal, v below it.
  */
 #include <math.h>
 #include <stdlib.h>
@@ -443,4 +450,80 @@ double oracle_zpotrf_backward_error(int n, const double* A0, int lda0, const dou
   if (den == 0.0L) return num == 0.0L ? 0.0 : INFINITY;
   const long double eps = ldexpl(1.0L, -53);
   return (double)(sqrtl(num) / ((long double)nb * sqrtl(den) * eps));
+}
+
+/* Householder QR of the m x n column-major a (leading dim lda), in place; tau[min(m,n)]. */
+void oracle_dgeqrf(int m, int n, double* a, int lda, double* tau) {
+  const int kmax = m < n ? m : n;
+  for (int k = 0; k < kmax; ++k) {
+    double* x = a + IDX(k, k, lda);
+    const double alpha = x[0];
+    double ss = 0.0;
+    for (int i = 1; i < m - k; ++i) ss = ss + x[i] * x[i];
+    const double xnorm = sqrt(ss);
+    if (xnorm == 0.0) {
+      tau[k] = 0.0;
+      continue; /* H = I: nothing to apply */
+    }
+    const double r = sqrt(alpha * alpha + xnorm * xnorm);
+    const double beta = alpha >= 0.0 ? -r : r;
+    tau[k] = (beta - alpha) / beta;
+    const double den = alpha - beta;
+    for (int i = 1; i < m - k; ++i) x[i] = x[i] / den;
+    x[0] = beta;
+    for (int j = k + 1; j < n; ++j) {
+      double* y = a + IDX(k, j, lda);
+      double w = y[0]; /* v_0 = 1 */
+      for (int i = 1; i < m - k; ++i) w = w + x[i] * y[i];
+      const double tw = tau[k] * w;
+      y[0] = y[0] - tw;
+      for (int i = 1; i < m - k; ++i) y[i] = y[i] - tw * x[i];
+    }
+  }
+}
+
+/* QR gates in long double: bwd = ||A - Q R||_F / (max(m,n) ||A||_F eps) and
+ * orth = ||Q^T Q - I||_F / (m eps), with Q = H_0 H_1 ... H_(k-1) (m x m) formed explicitly
+ * from the compact factor F (v below the diagonal, v_0 = 1) and tau; eps = 2^-53. */
+void oracle_geqrf_errors(int m, int n, const double* A0, int lda0, const double* F, int ldf,
+                         const double* tau, double* bwd, double* orth) {
+  const int kmax = m < n ? m : n;
+  *bwd = 0.0;
+  *orth = 0.0;
+  if (m <= 0 || n <= 0) return;
+  long double* Q = (long double*)calloc((size_t)m * m, sizeof(long double));
+  for (int i = 0; i < m; ++i) Q[(size_t)i * m + i] = 1.0L;
+  /* Q = H_0 ... H_(k-1): apply in reverse to I from the left */
+  for (int k = kmax - 1; k >= 0; --k) {
+    for (int j = 0; j < m; ++j) {
+      long double* q = Q + (size_t)j * m;
+      long double w = q[k];
+      for (int i = k + 1; i < m; ++i) w += (long double)F[IDX(i, k, ldf)] * q[i];
+      const long double tw = (long double)tau[k] * w;
+      q[k] -= tw;
+      for (int i = k + 1; i < m; ++i) q[i] -= tw * (long double)F[IDX(i, k, ldf)];
+    }
+  }
+  long double num = 0.0L, den = 0.0L;
+  for (int j = 0; j < n; ++j)
+    for (int i = 0; i < m; ++i) {
+      long double s = 0.0L;
+      for (int k = 0; k <= j && k < kmax; ++k) s += Q[(size_t)k * m + i] * (long double)F[IDX(k, j, ldf)];
+      const long double a = A0[IDX(i, j, lda0)];
+      num += (a - s) * (a - s);
+      den += a * a;
+    }
+  long double on = 0.0L;
+  for (int j = 0; j < m; ++j)
+    for (int i = 0; i < m; ++i) {
+      long double s = 0.0L;
+      for (int k = 0; k < m; ++k) s += Q[(size_t)i * m + k] * Q[(size_t)j * m + k];
+      const long double d = s - (i == j ? 1.0L : 0.0L);
+      on += d * d;
+    }
+  free(Q);
+  const long double eps = ldexpl(1.0L, -53);
+  const int mx = m > n ? m : n;
+  *bwd = den == 0.0L ? (num == 0.0L ? 0.0 : INFINITY) : (double)(sqrtl(num) / ((long double)mx * sqrtl(den) * eps));
+  *orth = (double)(sqrtl(on) / ((long double)m * eps));
 }

@@ -762,3 +762,54 @@ def test_zpotrf_info_and_backward_error_gate():
     D = Ae - Lp @ Lp.conj().T  # exact in double: entries are Gaussian integers +- 2^-40 terms
     exp = np.sqrt(np.sum(np.abs(D) ** 2)) / (n * np.sqrt(np.sum(np.abs(Ae) ** 2)) * 2.0 ** -53)
     assert oracle.zpotrf_backward_error(Ae, Lp, 0) == pytest.approx(exp, rel=1e-9)
+
+
+# ---------------------------------------------------------------- QR
+def test_qr_handworked_golden():
+    g = json.load(open(os.path.join(GOLD, "qr_handworked.json")))
+    for c in g["cases"]:
+        F, tau = oracle.dgeqrf(np.array(c["A"], dtype=np.float64))
+        Fx, tx = np.array(c["F"], dtype=np.float64), np.array(c["tau"], dtype=np.float64)
+        assert np.all(np.abs(F - Fx) <= 4 * 2.0 ** -52 * np.maximum(np.abs(Fx), 1e-300)), c["name"]
+        assert np.all(np.abs(tau - tx) <= 4 * 2.0 ** -52 * np.abs(tx)), c["name"]
+
+
+@pytest.mark.parametrize("m,n", [(1, 1), (2, 5), (7, 7), (50, 30), (30, 50), (130, 130), (257, 100)])
+def test_qr_matches_lapack_and_gates(m, n):
+    """Compact factor and tau within 1e-12 of LAPACK DGEQRF (OpenBLAS via scipy, MKL via torch);
+    reconstruction and orthogonality gates far below 10."""
+    import scipy.linalg
+    import torch
+    A = vbgen.g1_matrix(21, m * 1000 + n, m, n)
+    F, tau = oracle.dgeqrf(A)
+    (qr, tq), _ = scipy.linalg.qr(A, mode="raw")
+    scale = max(1.0, np.max(np.abs(qr)))
+    assert np.max(np.abs(F - qr)) <= 1e-12 * scale and np.max(np.abs(tau - tq[: len(tau)])) <= 1e-13
+    Ft, tt = torch.geqrf(torch.from_numpy(np.array(A)))
+    assert np.max(np.abs(F - Ft.numpy())) <= 1e-12 * scale
+    assert np.max(np.abs(tau - tt.numpy()[: len(tau)])) <= 1e-13
+    bwd, orth = oracle.geqrf_errors(A, F, tau)
+    assert bwd < 10 and orth < 10
+
+
+def test_qr_triangular_input_and_zero_columns():
+    """A column that is already zero below the diagonal: tau = 0, H = I, the column unchanged."""
+    A = np.triu(vbgen.g1_matrix(5, 1, 6, 6))
+    F, tau = oracle.dgeqrf(A)
+    assert np.array_equal(F, A) and not tau.any()
+    Z = np.zeros((4, 3))
+    F, tau = oracle.dgeqrf(Z)
+    assert not F.any() and not tau.any()
+
+
+def test_qr_gate_closed_form():
+    """Orthogonality gate: a single reflector for x = (3, 4) with tau perturbed by d gives
+    Q^T Q - I = (2 tau v^T v - 2) d v v^T + O(d^2) = 2 d v v^T (v = (1, 1/2)), so the gate reads
+    2 d ||v||^2 / (2 eps) = 2.5 d / (2 eps)."""
+    A = np.array([[3.0], [4.0]])
+    F, tau = oracle.dgeqrf(A)
+    b0, o0 = oracle.geqrf_errors(A, F, tau)
+    assert b0 < 1 and o0 < 1
+    d = 2.0 ** -40
+    _, o = oracle.geqrf_errors(A, F, tau + d)
+    assert o == pytest.approx(2.5 * d / (2 * 2.0 ** -53), rel=1e-3)
