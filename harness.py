@@ -299,3 +299,48 @@ def compare_zpotrf_with_oracle(A_in, L_gpu, info_gpu, single=False):
     tol = 8 * max(nb, 1) * 2.0 ** -24 if single else 1e-10
     res["ok"] = res["info_oracle"] == res["info_gpu"] and res["bwd"] <= 10.0 and res["rowscaled"] <= tol
     return res
+
+
+class QRBatch(LUBatch):
+    """A vbatched general-matrix problem for vbatched_dgeqrf: LUBatch's arena plus a tau arena
+    (min(m, n) doubles per matrix) and its device pointer array."""
+
+    def __init__(self, m, n, seed=1, ldda=None, device="cuda"):
+        super().__init__(m, n, seed=seed, ldda=ldda, device=device)
+        k = np.maximum(0, np.minimum(self.m, self.n)).astype(np.int64)
+        self.toff = np.concatenate([[0], np.cumsum((k + 31) // 32 * 32)[:-1]]).astype(np.int64)
+        self.tau = torch.full((int(self.toff[-1] + max(32, k[-1] + 32)),), float("nan"),
+                              dtype=torch.float64, device=device)
+        self.d_tau = torch.from_numpy((self.tau.data_ptr() + 8 * self.toff).astype(np.int64)).to(device)
+
+    def geqrf(self, max_m=None, max_n=None, stream=None, check=True):
+        from paper_conf_ipps_abdelfattahhtd16_b200 import vbatched_dgeqrf
+        mm = int(self.m.max()) if max_m is None else max_m
+        mn = int(self.n.max()) if max_n is None else max_n
+        return vbatched_dgeqrf(self.d_m, self.d_n, self.d_ptrs, self.d_ldda, self.d_tau, self.d_info,
+                               self.B, mm, mn, stream=stream, check=check)
+
+    def tau_of(self, i):
+        k = max(0, min(int(self.m[i]), int(self.n[i])))
+        return self.tau[int(self.toff[i]): int(self.toff[i]) + k].cpu().numpy()
+
+
+def compare_qr_with_oracle(A_in, F_gpu, tau_gpu):
+    """QR parity gates (DESIGN.md readings): reconstruction
+    ||A - QR||_F / (max(m,n) ||A||_F eps) <= 10 and orthogonality ||Q^T Q - I||_F / (m eps) <= 10
+    of the GPU's own factor (Q rebuilt from its v and tau), every entry of the compact factor
+    within 1e-10 of the oracle's scaled by the oracle row norm, tau within 1e-10."""
+    import oracle
+    m, n = A_in.shape
+    Fo, to = oracle.dgeqrf(A_in)
+    Fg = np.asfortranarray(F_gpu[:m, :n])
+    tg = np.asarray(tau_gpu, dtype=np.float64)
+    res = {"m": m, "n": n}
+    res["bwd"], res["orth"] = oracle.geqrf_errors(A_in, Fg, tg) if m and n else (0.0, 0.0)
+    rn = np.sqrt(np.sum(Fo * Fo, axis=1))
+    rn[rn == 0] = 1.0
+    res["rowscaled"] = float(np.max(np.abs(Fg - Fo) / rn[:, None])) if m and n else 0.0
+    res["tau_diff"] = float(np.max(np.abs(tg - to))) if len(to) else 0.0
+    res["ok"] = (res["bwd"] <= 10 and res["orth"] <= 10 and res["rowscaled"] <= 1e-10
+                 and res["tau_diff"] <= 1e-10)
+    return res

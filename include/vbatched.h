@@ -231,6 +231,27 @@ int vbatched_dgetrf(const int* d_m, const int* d_n, double* const* dA_array, con
                     vb_stream_t stream);
 
 /* ---------------------------------------------------------------------------------------
+ * vbatched_dgeqrf — FP64 variable-size batched Householder QR, A_i = Q_i R_i (SURVEY.md §8(f)
+ * NEXT-4; the QR extension of PAPER.md:2279-2285, built from the library's vbatched GEMM as the
+ * paper's separated design; LAPACK DGEQRF semantics).
+ *  d_m, d_n     [batchCount] rows / columns (device); rectangular allowed.
+ *  dA_array     [batchCount] device pointers, m_i x n_i column-major, ldda_i >= max(1, m_i). On
+ *               return R_i on and above the diagonal, the Householder vectors below it (v_k has
+ *               an implicit unit leading entry), Q_i = H_1 ... H_k, H_j = I - tau_j v_j v_j^T.
+ *  dtau_array   [batchCount] device pointers to min(m_i, n_i) doubles: the reflector scalars.
+ *  d_info       [batchCount] output: 0; -1 m_i < 0; -2 n_i < 0; -4 ldda_i < max(1, m_i); -9 m_i >
+ *               max_m or n_i > max_n (matrix untouched). QR itself never fails.
+ *  max_m, max_n bounds (host); max_m <= 1024 (panel rows in registers), larger returns -8.
+ * Reflectors: LAPACK DLARFG conventions (beta = -sign(alpha) sqrt(alpha^2 + ||x||^2), tau =
+ * (beta - alpha)/beta, v = x/(alpha - beta); ||x|| = 0 gives tau = 0). Internal workspace:
+ * batchCount x (16 max_m + 32 max_n + 256) doubles from the library's pool for the call.
+ * Returns 0 / -p (batchCount -7, max_m -8, max_n -9) / cudaError_t.
+ */
+int vbatched_dgeqrf(const int* d_m, const int* d_n, double* const* dA_array, const int* d_ldda,
+                    double* const* dtau_array, int* d_info, int batchCount, int max_m, int max_n,
+                    vb_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
  * Host helpers (pure host, deterministic, no CUDA).
  * vbatched_partition_lpt: flop-balanced multi-GPU sharding: longest
  *   processing time first on cost n^3/3 — sort by n descending (ties by index), assign

@@ -20,7 +20,7 @@ __all__ = [
     "vbatched_dpotrf_workspace_size", "vbatched_dpotrf_scan", "vbatched_dpotrf_factor", "vbatched_dgemm",
     "vbatched_dsyrk", "vbatched_dtrsm", "vbatched_partition_lpt", "vbatched_version",
     "vbatched_host_alloc", "vbatched_host_free", "vbatched_dpotrf_kernel_launches", "vbatched_dpotrf_kernel_names",
-    "vbatched_release_host_staging", "factor_kernel_names", "vbatched_dgetrf", "vbatched_zpotrf", "vbatched_cpotrf", "lib", "LIB_PATH", "VBatchedError",
+    "vbatched_release_host_staging", "factor_kernel_names", "vbatched_dgetrf", "vbatched_dgeqrf", "vbatched_zpotrf", "vbatched_cpotrf", "lib", "LIB_PATH", "VBatchedError",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -70,6 +70,7 @@ def lib() -> ctypes.CDLL:
         L.vbatched_dpotrf_kernel_names.restype = ctypes.c_char_p
         L.vbatched_zpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
         L.vbatched_cpotrf.argtypes = [_c, _vp, _vp, _vp, _vp, _i, _i, _vp]
+        L.vbatched_dgeqrf.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_dgetrf.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i, _i, _i, _vp]
         L.vbatched_release_host_staging.argtypes = []
         L.vbatched_release_host_staging.restype = _i
@@ -225,6 +226,15 @@ def vbatched_cpotrf(uplo, n, dA_array, ldda, info, batchCount, max_n, stream=Non
     rc = lib().vbatched_cpotrf(_ch(uplo), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(info),
                                int(batchCount), int(max_n), _stream(stream))
     return _check(rc, "vbatched_cpotrf") if check else rc
+
+
+def vbatched_dgeqrf(m, n, dA_array, ldda, dtau_array, info, batchCount, max_m, max_n, stream=None,
+                    check=True):
+    """vbatched Householder QR (include/vbatched.h): device arrays m, n, ldda, info (int32),
+    dA_array / dtau_array (int64 device pointers to the matrices / tau vectors)."""
+    rc = lib().vbatched_dgeqrf(_ptr(m), _ptr(n), _ptr(dA_array), _ptr(ldda), _ptr(dtau_array),
+                               _ptr(info), int(batchCount), int(max_m), int(max_n), _stream(stream))
+    return _check(rc, "vbatched_dgeqrf") if check else rc
 
 
 def vbatched_dgetrf(m, n, dA_array, ldda, dipiv_array, info, batchCount, max_m, max_n, stream=None,
