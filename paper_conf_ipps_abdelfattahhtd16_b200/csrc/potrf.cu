@@ -177,8 +177,8 @@ VB_DEVINL int potf2_regs_warp(double (&a)[NM], int nb, int lane, double* ws_, do
 // produces L21), the trailing 16x16 update C22 -= L21 L21^T on DMMA, POTF2 of C22.
 // sv/tv (>= 32 doubles) receive l_cc and 1/l_cc. Returns info.
 template <bool UP, typename E = double>
-VB_DEVINL int potf2_block32_impl(double* T, int ldt, int nb, int lane, E* Ag, int lda,
-                                 double* ws, double* sv, double* tv) {
+VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, E* Ag, int lda,
+                            double* ws, double* sv, double* tv) {
   const int nb1 = min(nb, 16), nb2 = nb - nb1;
   int info;
   {
@@ -250,15 +250,6 @@ VB_DEVINL int potf2_block32_impl(double* T, int ldt, int nb, int lane, E* Ag, in
   }
   __syncwarp();
   return info;
-}
-
-// Full 32-column tiles (every panel but a matrix's last) take a copy compiled for nb = 32: the
-// predicates on nb fold away (tools/chain_bench.cu: 7.5 K -> 5.6 K cycles alone).
-template <bool UP, typename E = double>
-VB_DEVINL int potf2_block32(double* T, int ldt, int nb, int lane, E* Ag, int lda, double* ws,
-                            double* sv, double* tv) {
-  if (nb == 32) return potf2_block32_impl<UP, E>(T, ldt, 32, lane, Ag, lda, ws, sv, tv);
-  return potf2_block32_impl<UP, E>(T, ldt, nb, lane, Ag, lda, ws, sv, tv);
 }
 
 // 32x32x32 DMMA products on a 4-warp group (wg = warp index 0..3): each warp owns a 16x16
@@ -415,12 +406,13 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
     // G here) and only ever feed output rows/columns that are never stored
     const int ra = (min(mrows, n - r0) + G - 1) / G * G;
     const int rb = (min(C::NB, n - j0) + G - 1) / G * G;
-    // the full barrier expects one arrival per producer lane (see the gather path below): lane
-    // 0 arrives with the transaction count, the others plainly
-    if (lane == 0)
-      mbar_arrive_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * (int)sizeof(E)));
+    // the full barrier expects 32 arrivals per phase (one per producer lane on the gather path
+    // below); here lane 0 posts the transaction bytes and the 32 arrivals itself
+    if (lane == 0) {  // the phase's transaction bytes, then all 32 expected arrivals at once
+      mbar_expect_tx(&s.full[st], (uint32_t)(C::KC * (ra + rb) * (int)sizeof(E)));
+      mbar_arrive_cnt(&s.full[st], 32);
+    }
     __syncwarp();
-    if (lane != 0) mbar_arrive(&s.full[st]);
     if (lane < C::KC) {
       // A rows stream (re-read only a panel later): evict first; the panel rows are re-read
       // for every row block of the panel: evict last (C5 DRAM traffic and time)
@@ -773,7 +765,7 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
   Ctrl* ctrl = const_cast<Ctrl*>(ctrl_c);
   if (threadIdx.x == 0) {
     for (int i = 0; i < C::STAGES; ++i) {
-      mbar_init(&s.full[i], 32);  // one arrival per producer lane
+      mbar_init(&s.full[i], 32);  // 32 arrivals per phase (see issue_chunk2)
       mbar_init(&s.empty[i], kV3Consumers);
     }
     mbar_init(&s.panel_done, kV3Consumers);
@@ -806,8 +798,10 @@ __global__ void __launch_bounds__(32 * (C::WARPS + 1), C::MINB)
   }
   // Chained without waiting (wait_upstream == 0): hold this grid's completion until the
   // upstream grid has completed, so that completion stays transitive along the PDL chain and
-  // stream successors (workspace free, caller kernels) see every earlier grid finished.
-  if (!wait_upstream && threadIdx.x == 0) pdl_wait();
+  // stream successors (workspace free, caller kernels) see every earlier grid finished. One
+  // thread of CTA 0 is enough (a grid completes when its last CTA exits); the other CTAs leave
+  // at once and free their SM slots for the next grid.
+  if (!wait_upstream && blockIdx.x == 0 && threadIdx.x == 0) pdl_wait();
 }
 
 // =======================================================================================
@@ -1107,7 +1101,7 @@ __global__ void __launch_bounds__(128, 4)
     if (role == 0 && lane == 0) s.info = 0;
     TL_END(role == 0 && lane == 0, t_tl, m, 22)
   }
-  if (!wait_upstream && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
+  if (!wait_upstream && blockIdx.x == 0 && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1167,7 +1161,7 @@ __global__ void __launch_bounds__(32 * kWarpsPerCta)
       potrf_warp_matrix<32, UP, E>(dA[m], n, ld, d_info + m, lane, s.w[wi], s.sv[wi], s.tv[wi]);
     TL_END(lane == 0, t_tl, m, 40)
   }
-  if (!wait_upstream && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
+  if (!wait_upstream && blockIdx.x == 0 && threadIdx.x == 0) pdl_wait();  // transitive completion (see blocked)
 }
 
 // Direct warp path for batches whose max_n <= 32 (no scan, no sort: with every matrix this
