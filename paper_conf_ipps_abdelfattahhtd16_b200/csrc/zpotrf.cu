@@ -252,22 +252,29 @@ VB_DEVINL void zpotrf_matrix(ZSmem& s, E2* __restrict__ A, int n, int ld, int* i
         s.info[p & 1] = info;
         if (info) *info_out = j0 + info;
       }
+      __syncwarp();  // the named barrier is entered by the whole, converged warp
       if (below) bar_group_arrive(1, 128);
     } else if (below) {
-      bool synced = false;
-      for (int st = p + warp; st < nstrip; st += 3) {
-        const int r0 = kZNB * st;
-        double ar[2][2][2], ai[2][2][2];
-        zstrip_init<UP, E2>(ar, ai, A, n, ld, r0, j0, kZNB, false, lane);
-        zstrip_kloop<UP, E2, false>(ar, ai, A, n, ld, r0, j0, 0, j0, lane);
-        if (!synced) {
-          bar_group(1, 128);
-          synced = true;
-        }
-        if (s.info[p & 1]) break;
-        zstrip_trsm_store<UP, E2>(s, ar, ai, A, n, ld, r0, j0, lane);
+      // the first strip's update overlaps warp 0's POTF2; every warp then meets the barrier at
+      // the same instruction (synccheck), and the remaining strips follow
+      const int first = p + warp;
+      double ar[2][2][2], ai[2][2][2];
+      if (first < nstrip) {
+        zstrip_init<UP, E2>(ar, ai, A, n, ld, kZNB * first, j0, kZNB, false, lane);
+        zstrip_kloop<UP, E2, false>(ar, ai, A, n, ld, kZNB * first, j0, 0, j0, lane);
       }
-      if (!synced) bar_group(1, 128);
+      __syncwarp();
+      bar_group(1, 128);
+      if (!s.info[p & 1]) {
+        for (int st = first; st < nstrip; st += 3) {
+          const int r0 = kZNB * st;
+          if (st != first) {
+            zstrip_init<UP, E2>(ar, ai, A, n, ld, r0, j0, kZNB, false, lane);
+            zstrip_kloop<UP, E2, false>(ar, ai, A, n, ld, r0, j0, 0, j0, lane);
+          }
+          zstrip_trsm_store<UP, E2>(s, ar, ai, A, n, ld, r0, j0, lane);
+        }
+      }
     }
     __syncthreads();  // the panel's L is stored before the next panel reads it; info settled
     if (s.info[p & 1]) return;

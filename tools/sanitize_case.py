@@ -28,6 +28,19 @@ def c1():
     assert np.all(db.info() == 0)
 
 
+def mixed_gather():
+    """The mixed batch with odd ldda only: every chunk of the blocked kernel goes through the
+    8-byte cp.async gather (generic-proxy writes racecheck can follow) instead of TMA."""
+    rng = np.random.default_rng(201)
+    n = np.concatenate([rng.integers(33, 129, 30), rng.integers(129, 501, 40)]).astype(np.int32)
+    for uplo in ("L", "U"):
+        db = DeviceBatch(n, seed=202, nonspd_mod=9, ldda_mode="odd").fill(poison=True, uplo=uplo)
+        db.dpotrf(uplo=uplo)
+        torch.cuda.synchronize()
+        exp = np.array([vbgen.nonspd_k(202, g, int(n[g])) if g % 9 == 8 else 0 for g in range(len(n))])
+        assert np.array_equal(db.info(), exp), uplo
+
+
 def mixed(scale=1):
     rng = np.random.default_rng(200)
     n = np.concatenate([rng.integers(1, 33, 60 // scale), rng.integers(33, 129, 80 // scale),
@@ -67,5 +80,5 @@ def z():
 
 
 if __name__ == "__main__":
-    {"c1": c1, "mixed": mixed, "mixed_small": lambda: mixed(4), "lu": lu, "z": z}[sys.argv[1]]()
+    {"c1": c1, "mixed": mixed, "mixed_small": lambda: mixed(4), "mixed_gather": mixed_gather, "lu": lu, "z": z}[sys.argv[1]]()
     print("case ok", sys.argv[1])
