@@ -17,6 +17,7 @@ namespace vb {
 
 constexpr int kScanThreads = 1024;
 constexpr int kKeys = 4096;  // sort keys: min(n, kKeys-1) (larger n share the top key)
+constexpr int kCache = 8;    // items per thread whose key stays in registers (batch <= 8192)
 
 __global__ void __launch_bounds__(kScanThreads, 1)
     scan_bin_kernel(const int* __restrict__ d_n, const int* __restrict__ d_ldda,
@@ -31,8 +32,32 @@ __global__ void __launch_bounds__(kScanThreads, 1)
   for (int k = tid; k < kKeys; k += kScanThreads) hist[k] = 0;
   __syncthreads();
 
+  // The first kCache items of each thread keep their sort key in registers for the scatter
+  // pass (batch <= 8192 needs no second read of n / info); the loads of a thread's items are
+  // issued together (unrolled) so their latencies overlap. key < 0: not sorted (invalid, n=0).
+  int key[kCache];
   int mymax = 0;
-  for (int i = tid; i < batch; i += kScanThreads) {
+#pragma unroll
+  for (int u = 0; u < kCache; ++u) {
+    const int i = tid + u * kScanThreads;
+    key[u] = -1;
+    if (i < batch) {
+      const int n = d_n[i], ld = d_ldda[i];
+      int code = 0;
+      if (n < 0) code = -2;
+      else if (ld < (n > 1 ? n : 1)) code = -4;
+      else if (check_max && n > max_n) code = -7;
+      d_info[i] = code;
+      if (code == 0 && n > 0) {
+        key[u] = n < kKeys ? n : kKeys - 1;
+        mymax = n > mymax ? n : mymax;
+      }
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < kCache; ++u)
+    if (key[u] >= 0) atomicAdd(&hist[key[u]], 1);
+  for (int i = tid + kCache * kScanThreads; i < batch; i += kScanThreads) {
     const int n = d_n[i], ld = d_ldda[i];
     int code = 0;
     if (n < 0) code = -2;
@@ -97,7 +122,10 @@ __global__ void __launch_bounds__(kScanThreads, 1)
     ctrl->max_n = wmax[0];
   }
   __syncthreads();
-  for (int i = tid; i < batch; i += kScanThreads) {
+#pragma unroll
+  for (int u = 0; u < kCache; ++u)
+    if (key[u] >= 0) order[atomicAdd(&hist[key[u]], 1)] = tid + u * kScanThreads;
+  for (int i = tid + kCache * kScanThreads; i < batch; i += kScanThreads) {
     const int n = d_n[i];
     // re-derive validity exactly as above (info was written by this thread)
     if (d_info[i] == 0 && n > 0) {
