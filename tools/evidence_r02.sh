@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-2 evidence on the GPU box -> gpurun_out/ev2/ (summaries copied to profiles/r02/).
 cd "$(dirname "$0")/.."
-O=gpurun_out/ev2; mkdir -p $O
+O=gpurun_out/ev3; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $O/smi.txt
 timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider -s > $O/pytest_gpu.txt 2>&1; echo "rc=$?" >> $O/pytest_gpu.txt
