@@ -290,7 +290,9 @@ struct Cfg2 {
   static constexpr int LDA = MB + PAD, LDB = NB + PAD, LDT = NB + 4;
   static constexpr int G = 16 / (int)sizeof(E_);  // elements per 16 bytes (bulk-copy granule)
 };
-using Cfg64d = Cfg2<64, 16, 2, 3, 4>;  // v3, 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer
+// 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer; ring of 2 x 16-column chunks (measured
+// against 3 x 8 and 4 x 8: C5 154.4 / 160.5 vs 152.3 ms, the per-chunk barrier cost dominates)
+using Cfg64d = Cfg2<64, 16, 2, 3, 4>;
 using Cfg64s = Cfg2<64, 16, 2, 3, 4, float>;  // the same for FP32 storage (SPOTRF)
 
 template <class C>
@@ -429,16 +431,17 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
     // 'U': L's rows are contiguous in storage (16 k-values of one row = 128 B), 16 lanes per
     // row. Each lane's arrival on the full barrier is its cp.async.mbarrier.arrive.noinc,
     // triggered when all of that lane's copies have landed (32 expected arrivals per phase).
-    static_assert(C::KC == 16 && C::MB % 32 == 0 && C::NB % 32 == 0, "copy shapes");
+    static_assert((C::KC == 8 || C::KC == 16) && C::MB % 32 == 0 && C::NB % 32 == 0, "copy shapes");
     if (UP) {
-      const int c = lane & 15;
+      constexpr int RS = 32 / C::KC;  // rows per pass (KC lanes per row)
+      const int c = lane % C::KC;
 #pragma unroll 4
-      for (int r = lane >> 4; r < C::MB; r += 2) {
+      for (int r = lane / C::KC; r < C::MB; r += RS) {
         const bool p = r < mrows && r0 + r < n;
         cp_async_e<E>(&s.a[st][c][r], A + (p ? (size_t)(r0 + r) * ld + k0 + c : 0), p);
       }
 #pragma unroll 4
-      for (int r = lane >> 4; r < C::NB; r += 2) {
+      for (int r = lane / C::KC; r < C::NB; r += RS) {
         const bool p = j0 + r < n;
         cp_async_e<E>(&s.b[st][c][r], A + (p ? (size_t)(j0 + r) * ld + k0 + c : 0), p);
       }

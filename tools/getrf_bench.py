@@ -1,5 +1,6 @@
-"""vbatched_dgetrf throughput: one JSON line per workload.
-python tools/getrf_bench.py [count] [nmax] ...  (square matrices, n ~ U{1..nmax}, seeded)
+"""vbatched_dgetrf / vbatched_dgeqrf throughput: one JSON line per
+workload. python tools/getrf_bench.py [count] [nmax] ...  (square matrices, n ~ U{1..nmax});
+OP=qr selects vbatched_dgeqrf (LAPACK DGEQRF flops for m = n: 4n^3/3 + n^2 + 14n/3... ~ 4n^3/3).
 GFLOP/s counts the LAPACK DGETRF flops of each matrix (m n^2 - n^3/3 - n^2/2 + 5n/6 for m = n:
 2n^3/3 - n^2/2 + 5n/6); timing: CUDA events around the call, inputs restored and L2 flushed
 before each of 10 timed reps (3 warm-up). The roofline denominator is the measured FP64 DMMA
@@ -13,11 +14,15 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-from harness import LUBatch  # noqa: E402
+from harness import LUBatch, QRBatch  # noqa: E402
+
+QR = os.environ.get("OP") == "qr"
 
 
 def flops(n):
     n = n.astype(np.float64)
+    if QR:
+        return float(np.sum(4 * n ** 3 / 3 + n ** 2 + 14 * n / 3))
     return float(np.sum(2 * n ** 3 / 3 - n ** 2 / 2 + 5 * n / 6))
 
 
@@ -26,7 +31,7 @@ peak = json.load(open(os.path.join(os.path.dirname(__file__), "..", "profiles", 
 for cnt, nmax in zip(args[0::2], args[1::2]):
     cnt, nmax = int(cnt), int(nmax)
     n = np.random.default_rng(nmax).integers(1, nmax + 1, cnt).astype(np.int32)
-    lb = LUBatch(n, n, seed=13).fill()
+    lb = (QRBatch if QR else LUBatch)(n, n, seed=13).fill()
     pristine = lb.arena.clone()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     times = []
@@ -35,7 +40,7 @@ for cnt, nmax in zip(args[0::2], args[1::2]):
         flush.fill_(1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        lb.getrf()
+        lb.geqrf() if QR else lb.getrf()
         e1.record()
         torch.cuda.synchronize()
         if rep >= 3:
@@ -47,9 +52,9 @@ for cnt, nmax in zip(args[0::2], args[1::2]):
     idx = np.arange(0, cnt, max(1, cnt // 100))
     t0 = time.perf_counter()
     for i in idx:
-        oracle.dgetrf(lb.inputs[int(i)])
+        (oracle.dgeqrf if QR else oracle.dgetrf)(lb.inputs[int(i)])
     tc = time.perf_counter() - t0
-    line = {"op": "vbatched_dgetrf", "workload": f"{cnt} x U{{1..{nmax}}} square, g1 values",
+    line = {"op": "vbatched_dgeqrf" if QR else "vbatched_dgetrf", "workload": f"{cnt} x U{{1..{nmax}}} square, g1 values",
             "value": fl / t / 1e9, "unit": "GFLOP/s", "ms": t * 1e3, "best_ms": min(times) * 1e3,
             "roofline": {"bound": "tensor", "achieved": fl / t / 1e12, "peak": peak,
                          "frac": fl / t / 1e12 / peak, "unit": "TFLOP/s"},
