@@ -978,7 +978,7 @@ VB_DEVINL void small_trsm_store(SmallSmem& s, double (&acc)[4][4][2], E* __restr
 // bar0 = inv ready (D -> O), bar0+1 = tile ready (O -> D), bar0+2 = inverse free (O -> D).
 template <bool UP, typename E>
 VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A, int n, int ld,
-                            int* info_out, int bar0) {
+                            int* info_out, int bar0, int bar_lb) {
   const int g = lane >> 2, q = lane & 3;
   const int npan = (n + 31) / 32;
   if (role == 0) {
@@ -1006,6 +1006,18 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
       if (lane == 0) s.info = 0;
       bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready (s.T is free again)
       pending_free = true;
+      // The off-diagonal warp carries every other update and is the pair's bottleneck (ncu: the
+      // diagonal warp waits ~37 % of its time for the next tile); the diagonal warp takes the
+      // panel's last 32-row block when the panel has >= 3 blocks, while it would wait anyway.
+      const int nblk = (n - j0 + 31) / 32;
+      if (nblk >= 3) {
+        double acc[4][4][2];
+        const int r0 = j0 + 32 * (nblk - 1);
+        small_panel_update<UP>(acc, A, n, ld, r0, j0, 32, false, lane);
+        small_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
+        __syncwarp();
+        bar_group_arrive(bar_lb, 64);  // last block of panel p stored
+      }
     }
   } else {
     {  // tile of panel 0: A's diagonal block as it is
@@ -1025,6 +1037,8 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
       const int j0 = 32 * p;
       const int nblk = (n - j0 + 31) / 32;
       double acc[4][4][2];
+      // panel p-1's last block was the diagonal warp's: its stores precede any read of them here
+      if (p > 0 && nblk + 1 >= 3) bar_group(bar_lb, 64);
       small_panel_update<UP>(acc, A, n, ld, j0 + 32, j0, 32, false, lane);
       bar_group(bar0, 64);  // inv(L11) of panel p (or the failure)
       if (s.info) break;
@@ -1061,7 +1075,8 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
         __syncwarp();
         bar_group_arrive(bar0 + 1, 64);  // tile of panel p+1 ready
       }
-      for (int b = 2; b < nblk; ++b) {
+      const int bend = nblk >= 3 ? nblk - 1 : nblk;  // the last block is the diagonal warp's
+      for (int b = 2; b < bend; ++b) {
         small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
         small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
       }
@@ -1099,7 +1114,7 @@ __global__ void __launch_bounds__(128, 4)
     if (it >= count) break;
     const int m = order[start + it];
     TL_BEGIN(t_tl)
-    la_matrix_v2<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0);
+    la_matrix_v2<UP, E>(s, role, lane, dA[m], d_n[m], d_ldda[m], d_info + m, bar0, 9 + pair);
     bar_group(tsync, 64);
     if (role == 0 && lane == 0) s.info = 0;
     TL_END(role == 0 && lane == 0, t_tl, m, 22)
