@@ -1006,17 +1006,22 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
       if (lane == 0) s.info = 0;
       bar_group_arrive(bar0, 64);  // inv(L11) of panel p is ready (s.T is free again)
       pending_free = true;
-      // The off-diagonal warp carries every other update and is the pair's bottleneck (ncu: the
-      // diagonal warp waits ~37 % of its time for the next tile); the diagonal warp takes the
-      // panel's last 32-row block when the panel has >= 3 blocks, while it would wait anyway.
+      // The off-diagonal warp carried every other update and was the pair's bottleneck (ncu: the
+      // diagonal warp waited ~37 % of its time for the next tile); the diagonal warp now takes
+      // the panel's blocks from the second one below the diagonal on (every block but block 1,
+      // whose rows form the next tile), while it would wait anyway: C2 121 -> 117 us with the
+      // last block only, -> 113 us with all of them (tools/ab_time.py).
       const int nblk = (n - j0 + 31) / 32;
       if (nblk >= 3) {
-        double acc[4][4][2];
-        const int r0 = j0 + 32 * (nblk - 1);
-        small_panel_update<UP>(acc, A, n, ld, r0, j0, 32, false, lane);
-        small_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
+        const int b0 = nblk >= 4 ? nblk - 2 : nblk - 1;
+        for (int b = b0; b < nblk; ++b) {
+          double acc[4][4][2];
+          const int r0 = j0 + 32 * b;
+          small_panel_update<UP>(acc, A, n, ld, r0, j0, 32, false, lane);
+          small_trsm_store<UP>(s, acc, A, n, ld, r0, j0, lane);
+        }
         __syncwarp();
-        bar_group_arrive(bar_lb, 64);  // last block of panel p stored
+        bar_group_arrive(bar_lb, 64);  // last block(s) of panel p stored
       }
     }
   } else {
@@ -1075,7 +1080,7 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
         __syncwarp();
         bar_group_arrive(bar0 + 1, 64);  // tile of panel p+1 ready
       }
-      const int bend = nblk >= 3 ? nblk - 1 : nblk;  // the last block is the diagonal warp's
+      const int bend = nblk >= 4 ? nblk - 2 : (nblk >= 3 ? nblk - 1 : nblk);  // diagonal warp's
       for (int b = 2; b < bend; ++b) {
         small_panel_update<UP>(acc, A, n, ld, j0 + 32 * b, j0, 32, false, lane);
         small_trsm_store<UP>(s, acc, A, n, ld, j0 + 32 * b, j0, lane);
