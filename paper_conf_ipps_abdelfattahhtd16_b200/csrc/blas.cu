@@ -220,6 +220,30 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
     __syncthreads();  // the next tile's prologue refills stages 0 and 1
     double* C = a.C[mi];
     const int ldc = a.ldc[mi];
+    // Epilogue in two passes: every load of C first (all in flight together), then every store.
+    // As one read-modify-write per element the loads serialise behind the stores (the compiler
+    // cannot move a load of C past a store to C): one memory round trip per element, most of a
+    // tile's time for small k (the rank-16 trailing updates of GETRF/GEQRF).
+    if (a.beta != 0.0) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 4; ++y)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int r = r0 + wr + x * 8 + g, c = c0 + wc + y * 8 + 2 * q + h;
+            const bool p = r < m && c < n && !(a.mode == kSyrkLower && r < c) &&
+                           !(a.mode == kSyrkUpper && r > c);
+            acc[x][y][h] = a.alpha * acc[x][y][h] + (p ? a.beta * C[(size_t)c * ldc + r] : 0.0);
+          }
+    } else {
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 4; ++y)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) acc[x][y][h] *= a.alpha;
+    }
 #pragma unroll
     for (int x = 0; x < 4; ++x)
 #pragma unroll
@@ -230,9 +254,7 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
           if (r >= m || c >= n) continue;
           if (a.mode == kSyrkLower && r < c) continue;
           if (a.mode == kSyrkUpper && r > c) continue;
-          double* pc = C + (size_t)c * ldc + r;
-          const double v = a.alpha * acc[x][y][h];
-          *pc = (a.beta == 0.0) ? v : fma(a.beta, *pc, v);
+          C[(size_t)c * ldc + r] = acc[x][y][h];
         }
   }
 }
@@ -287,7 +309,7 @@ __device__ __forceinline__ void trsm_stage(TrsmSmem& s, int st, const BlasArgs& 
   for (int e = 0; e < (kTC * kBT) / kGThreads; ++e) {
     const int idx = tid + e * kGThreads;
     // contiguous direction of the storage view first: rows for B, k for B^T (side 'L')
-    const int k = idx / kBT, i = idx % kBT;
+    const int k = a.bt ? idx % kTC : idx / kBT, i = a.bt ? idx / kTC : idx % kBT;
     const bool p = (k0 + k < kend) && (r0 + i < m);
     cp_async8(&s.u.ring.xa[st][k][i], B + (p ? bix(a.bt, r0 + i, k0 + k, ldb) : 0), p);
   }
@@ -327,6 +349,24 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
     for (int step = 0; step < nbk; ++step) {
       const int J = a.tlower ? nbk - 1 - step : step;
       const int c0 = J * kTW, w = min(kTW, n - c0);
+      // B_J and T_JJ are read into registers before the accumulation loop (neither is written
+      // before this step's end), so these 24 loads per thread overlap it instead of running as
+      // dependent round trips after it. Index order: the storage view's contiguous direction
+      // across the lanes (rows of B; for B^T the columns of B_J).
+      constexpr int kBE = (kTW * kBT) / kGThreads, kTE = (kTW * kTW) / kGThreads;
+      double bv[kBE], tjj[kTE];
+#pragma unroll
+      for (int e = 0; e < kBE; ++e) {
+        const int idx = tid + e * kGThreads;
+        const int k = a.bt ? idx % kTW : idx / kBT, i = a.bt ? idx / kTW : idx % kBT;
+        bv[e] = (k < w && r0 + i < m) ? B[bix(a.bt, r0 + i, c0 + k, ldb)] : 0.0;
+      }
+#pragma unroll
+      for (int e = 0; e < kTE; ++e) {
+        const int idx = tid + e * kGThreads;
+        const int j = a.ta ? idx % kTW : idx / kTW, i = a.ta ? idx / kTW : idx % kTW;
+        tjj[e] = (i < w && j < w) ? t_elem(a, A, lda, c0 + i, c0 + j) : (i == j ? 1.0 : 0.0);
+      }
       double acc[4][2][2];
 #pragma unroll
       for (int x = 0; x < 4; ++x)
@@ -372,17 +412,19 @@ __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* 
           for (int h = 0; h < 2; ++h) s.u.e.x[wc + y * 8 + 2 * q + h][wr + x * 8 + g] = -acc[x][y][h];
       // TRTRI input L (lower, L[r][c] at d[c][r]): L = T_JJ when T is lower, L = T_JJ^T when
       // it is upper (then inv(L)^T = inv(T_JJ) comes out of TRTRI directly)
-      for (int idx = tid; idx < kTW * kTW; idx += kGThreads) {
-        const int j = idx / kTW, i = idx % kTW;
-        const double v = (i < w && j < w) ? t_elem(a, A, lda, c0 + i, c0 + j) : (i == j ? 1.0 : 0.0);
-        if (a.tlower) s.d[j][i] = v;
-        else s.d[i][j] = v;
+#pragma unroll
+      for (int e = 0; e < kTE; ++e) {
+        const int idx = tid + e * kGThreads;
+        const int j = a.ta ? idx % kTW : idx / kTW, i = a.ta ? idx / kTW : idx % kTW;
+        if (a.tlower) s.d[j][i] = tjj[e];
+        else s.d[i][j] = tjj[e];
       }
       __syncthreads();
-      for (int idx = tid; idx < kTW * kBT; idx += kGThreads) {
-        const int k = idx / kBT, i = idx % kBT;
-        const double bv = (k < w && r0 + i < m) ? B[bix(a.bt, r0 + i, c0 + k, ldb)] : 0.0;
-        s.u.e.x[k][i] = fma(a.alpha, bv, s.u.e.x[k][i]);
+#pragma unroll
+      for (int e = 0; e < kBE; ++e) {
+        const int idx = tid + e * kGThreads;
+        const int k = a.bt ? idx % kTW : idx / kBT, i = a.bt ? idx / kTW : idx % kBT;
+        s.u.e.x[k][i] = fma(a.alpha, bv[e], s.u.e.x[k][i]);
       }
       // inv(T_JJ) by warp 0: 8x8 substitution + recursive doubling on DMMA (trtri32_dmma_warp)
       // into the B-operand layout INV[k][n] = inv(L)[n][k]; for a lower T that is inv(T)^T,

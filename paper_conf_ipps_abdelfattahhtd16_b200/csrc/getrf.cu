@@ -7,10 +7,11 @@
 // Built the paper's "separated" way: a host loop over panels of NB columns,
 // each step = an aux kernel that derives the per-matrix sub-problem sizes and pointers on the
 // GPU (the size arrays live there), a fused panel kernel (getf2 with partial
-// pivoting, rows in registers), the row interchanges on the other columns (laswp), and then
-// the SAME vbatched TRSM and GEMM kernels that vbatched_dtrsm / vbatched_dgemm export:
-//   A12 <- L11^-1 A12   (vbatched TRSM, side L, lower, unit diagonal)
+// pivoting, rows in registers), the row interchanges on the columns right of the panel fused
+// with the unit-lower solve A12 <- L11^-1 A12 (laswp + trsm, one warp per column), and then the
+// SAME vbatched GEMM kernel that vbatched_dgemm exports:
 //   A22 <- A22 - A21 A12 (vbatched GEMM, DMMA)
+// The interchanges on the columns left of each panel are applied once after the last step.
 // Matrices whose panel is exhausted get size 0 in the step arrays and cost no tiles.
 #include <algorithm>
 
@@ -193,16 +194,47 @@ __global__ void __launch_bounds__(kLuThreads)
   }
 }
 
-// Row interchanges of the step's pivots on the columns outside the panel (LAPACK DLASWP on
-// columns 0..j-1 and j+pn..n-1). The pn sequential swaps only move rows of the set
-// S = {j..j+pn-1} u {ipiv targets} (<= 2 pn <= 64 rows); their composition is a permutation pi
-// of S, built once per matrix in shared memory. Then one warp per column: each lane loads two
-// rows of S (one coalesced run j..j+pn-1, the rest scattered), and writes row S[t] with the
-// value of row pi(S[t]) taken by a shuffle — one gather and one scatter per column instead of
-// 2 pn dependent strided accesses.
+// The composition of a step's pn sequential interchanges (LAPACK DLASWP order, ipiv[k] >= k)
+// only moves rows of the set S = {j..j+pn-1} u {ipiv targets} (<= 2 pn <= 64 rows): a
+// permutation of S, built by one thread. Slot t holds row srow[t]; after the interchanges row
+// srow[t] holds the old value of row srow[ssrc[t]]. Slots 0..pn-1 are rows j..j+pn-1.
+__device__ int lu_step_perm(const int* ip, int j, int pn, int* srow, int* ssrc) {
+  int cnt = pn;
+  int cur[2 * kLuNB];  // cur[t]: slot whose original value currently sits in S[t]
+  for (int t = 0; t < pn; ++t) {
+    srow[t] = j + t;
+    cur[t] = t;
+  }
+  for (int k = 0; k < pn; ++k) {
+    const int r2 = ip[k] - 1;
+    int t2 = -1;
+    for (int t = 0; t < cnt; ++t)
+      if (srow[t] == r2) t2 = t;
+    if (t2 < 0) {
+      t2 = cnt++;
+      srow[t2] = r2;
+      cur[t2] = t2;
+    }
+    const int x = cur[k];
+    cur[k] = cur[t2];
+    cur[t2] = x;
+  }
+  for (int t = 0; t < cnt; ++t) ssrc[t] = cur[t];
+  return cnt;
+}
+
+// Row interchanges of the step's pivots on the columns right of the panel, fused with the
+// triangular solve A12 <- L11^-1 A12 (DTRSM 'L','L','N','U', PAPER.md:760-812 reused as a
+// fused step). One warp per column: each lane loads two rows of S (one coalesced run
+// j..j+pn-1, the rest scattered), takes the value of row pi(S[t]) by a shuffle, and lanes
+// 0..pn-1 (the rows j..j+pn-1, now A12's column) run the unit-lower forward substitution with
+// L11 held in registers (lane t: L(j+t, j+k), k < t), one shuffle per column of L11. The
+// columns left of the panel are not touched here: their interchanges are applied once, after
+// the last step (lu_laswp_left_kernel).
 __global__ void __launch_bounds__(256)
-    lu_laswp_kernel(LuStep st, double* const* __restrict__ dA, const int* __restrict__ d_n,
-                    const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv, int batch, int j) {
+    lu_laswp_trsm_kernel(LuStep st, double* const* __restrict__ dA, const int* __restrict__ d_n,
+                         const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv, int batch,
+                         int j) {
   __shared__ int srow[2 * kLuNB];  // S
   __shared__ int ssrc[2 * kLuNB];  // for slot t: the slot whose old value moves to S[t]
   __shared__ int s_cnt;
@@ -211,46 +243,83 @@ __global__ void __launch_bounds__(256)
     const int pn = st.pn[i];
     if (pn <= 0) continue;
     const int n = d_n[i], ld = d_ld[i];
+    if (j + pn >= n) continue;
     double* A = dA[i];
-    const int* ip = d_ipiv[i] + j;
-    if (threadIdx.x == 0) {
-      // slots 0..pn-1: rows j..j+pn-1; further slots: targets outside that range
-      int cnt = pn;
-      int cur[2 * kLuNB];  // cur[t]: slot whose original value currently sits in S[t]
-      for (int t = 0; t < pn; ++t) {
-        srow[t] = j + t;
-        cur[t] = t;
-      }
-      for (int k = 0; k < pn; ++k) {
-        const int r2 = ip[k] - 1;
-        int t2 = -1;
-        for (int t = 0; t < cnt; ++t)
-          if (srow[t] == r2) t2 = t;
-        if (t2 < 0) {
-          t2 = cnt++;
-          srow[t2] = r2;
-          cur[t2] = t2;
-        }
-        const int x = cur[k];
-        cur[k] = cur[t2];
-        cur[t2] = x;
-      }
-      for (int t = 0; t < cnt; ++t) ssrc[t] = cur[t];
-      s_cnt = cnt;
-    }
+    if (threadIdx.x == 0) s_cnt = lu_step_perm(d_ipiv[i] + j, j, pn, srow, ssrc);
     __syncthreads();
     const int cnt = s_cnt;
     const int r_lo = lane < cnt ? srow[lane] : 0, r_hi = lane + 32 < cnt ? srow[lane + 32] : 0;
     const int f_lo = lane < cnt ? ssrc[lane] : 0, f_hi = lane + 32 < cnt ? ssrc[lane + 32] : 0;
-    for (int c = warp; c < n; c += nw) {
-      if (c >= j && c < j + pn) continue;
+    const double* L11 = A + (size_t)j * ld + j;
+    double l11[kLuNB];
+#pragma unroll
+    for (int k = 0; k < kLuNB; ++k) l11[k] = (k < lane && lane < pn) ? L11[(size_t)k * ld + lane] : 0.0;
+    for (int c = j + pn + warp; c < n; c += nw) {
       double* col = A + (size_t)c * ld;
       const double v_lo = lane < cnt ? col[r_lo] : 0.0;
       const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
       const double a_lo = __shfl_sync(kFull, v_lo, f_lo & 31), b_lo = __shfl_sync(kFull, v_hi, f_lo & 31);
       const double a_hi = __shfl_sync(kFull, v_lo, f_hi & 31), b_hi = __shfl_sync(kFull, v_hi, f_hi & 31);
-      if (lane < cnt) col[r_lo] = f_lo < 32 ? a_lo : b_lo;
+      double x = f_lo < 32 ? a_lo : b_lo;
+#pragma unroll
+      for (int k = 0; k < kLuNB - 1; ++k) {
+        const double xk = __shfl_sync(kFull, x, k);
+        x = fma(-l11[k], xk, x);  // l11[k] = 0 for lanes <= k and lanes >= pn
+      }
+      if (lane < cnt) col[r_lo] = x;
       if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
+    }
+    __syncthreads();
+  }
+}
+
+// The interchanges on the columns left of each panel, deferred to the end (pure data movement:
+// the same result as applying them step by step, LAPACK DGETRF's DLASWP on columns 0..j-1).
+// Columns of 16-column block b see the interchanges of every later step; their composition
+// src_b (row r receives the value of row src_b[r]) is built backwards, src_b = sigma_{b+1} o
+// src_{b+1}, with sigma_{b+1} the permutation of step b+1's set S. Each column segment below
+// the block is read once (coalesced) into shared memory and only the moved rows are written.
+__global__ void __launch_bounds__(256)
+    lu_laswp_left_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                         double* const* __restrict__ dA, const int* __restrict__ d_ld,
+                         int* const* __restrict__ d_ipiv, const int* __restrict__ d_info, int batch) {
+  __shared__ int src[kLuThreads * kLuMaxRPT];
+  __shared__ double buf[kLuThreads * kLuMaxRPT];
+  __shared__ int srow[2 * kLuNB], ssrc[2 * kLuNB];
+  __shared__ int s_cnt;
+  const int tid = threadIdx.x;
+  for (int i = blockIdx.x; i < batch; i += gridDim.x) {
+    if (d_info[i] < 0) continue;
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    const int kmax = m < n ? m : n;
+    const int nblk = (kmax + kLuNB - 1) / kLuNB;
+    if (nblk < 2) continue;
+    double* A = dA[i];
+    const int* ip = d_ipiv[i];
+    for (int r = tid; r < m; r += blockDim.x) src[r] = r;
+    for (int b = nblk - 2; b >= 0; --b) {
+      const int j = (b + 1) * kLuNB, pn = min(kLuNB, kmax - j);
+      __syncthreads();  // src complete, previous block's buf reads done
+      if (tid == 0) s_cnt = lu_step_perm(ip + j, j, pn, srow, ssrc);
+      __syncthreads();
+      const int cnt = s_cnt;
+      for (int r = j + tid; r < m; r += blockDim.x) {
+        const int x = src[r];
+        int y = x;
+        for (int t = 0; t < cnt; ++t)
+          if (srow[t] == x) y = srow[ssrc[t]];
+        src[r] = y;
+      }
+      for (int c = b * kLuNB; c < j; ++c) {
+        double* col = A + (size_t)c * ld;
+        __syncthreads();  // src updated; buf free
+        for (int r = j + tid; r < m; r += blockDim.x) buf[r] = col[r];
+        __syncthreads();
+        for (int r = j + tid; r < m; r += blockDim.x) {
+          const int y = src[r];
+          if (y != r) col[r] = buf[y];
+        }
+      }
     }
     __syncthreads();
   }
@@ -298,19 +367,20 @@ int getrf_impl(const int* d_m, const int* d_n, double* const* dA, const int* d_l
     else if (rows <= 2 * kLuThreads) e = launch_panel<2>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
     else e = launch_panel<4>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
     if (e != cudaSuccess) break;
-    lu_laswp_kernel<<<pg, 256, 0, stream>>>(st, dA, d_n, d_ld, d_ipiv, batch, j);
-    if ((e = cudaGetLastError()) != cudaSuccess) break;
     if (j + kLuNB < max_n) {
-      int rc = trsm_launch('L', 'L', 'N', 'U', st.pn, st.rn, 1.0, st.P, d_ld, st.A12, d_ld, batch,
-                           kLuNB, max_n, stream);
-      if (rc == 0)
-        rc = gemm_launch('N', 'N', st.bm, st.rn, st.pn, -1.0, st.A21, d_ld, st.A12, d_ld, 1.0,
-                         st.A22, d_ld, batch, max_m, max_n, kLuNB, stream);
+      lu_laswp_trsm_kernel<<<pg, 256, 0, stream>>>(st, dA, d_n, d_ld, d_ipiv, batch, j);
+      if ((e = cudaGetLastError()) != cudaSuccess) break;
+      int rc = gemm_launch('N', 'N', st.bm, st.rn, st.pn, -1.0, st.A21, d_ld, st.A12, d_ld, 1.0,
+                           st.A22, d_ld, batch, max_m, max_n, kLuNB, stream);
       if (rc != 0) {
         e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
         break;
       }
     }
+  }
+  if (e == cudaSuccess && kmax > kLuNB) {
+    lu_laswp_left_kernel<<<pg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_ipiv, d_info, batch);
+    e = cudaGetLastError();
   }
   cudaError_t e2 = ws_free(ws, stream);
   return (int)(e != cudaSuccess ? e : e2);
