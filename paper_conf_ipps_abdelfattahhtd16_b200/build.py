@@ -11,6 +11,7 @@ import glob
 import os
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
@@ -37,10 +38,26 @@ def build_lib(force: bool = False, verbose: bool = False) -> str:
     deps = srcs + glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h")) + \
         [os.path.join(ROOT, "include", "vbatched.h")]
     if force or _stale(LIB, deps):
-        cmd = [NVCC, *ARCH, *COMMON, "-I", os.path.join(ROOT, "include"), "-o", LIB, *srcs]
-        if verbose:
-            cmd.insert(1, "-Xptxas=-v")
-        subprocess.check_call(cmd)
+        # one object per translation unit, compiled in parallel (whole-program device code stays
+        # per file: no relocatable device code, the units share only inline headers), then linked
+        objdir = os.path.join(PKG, "build")
+        os.makedirs(objdir, exist_ok=True)
+        cflags = [f for f in COMMON if f not in ("-shared",)]
+        inc = ["-I", os.path.join(ROOT, "include")]
+        hdrs = [d for d in deps if not d.endswith(".cu")]
+
+        def compile_one(src: str) -> str:
+            obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+            if force or _stale(obj, [src, *hdrs]):
+                cmd = [NVCC, *ARCH, *cflags, *inc, "-c", src, "-o", obj]
+                if verbose:
+                    cmd.insert(1, "-Xptxas=-v")
+                subprocess.check_call(cmd)
+            return obj
+
+        with ThreadPoolExecutor(max_workers=min(len(srcs), os.cpu_count() or 1)) as ex:
+            objs = list(ex.map(compile_one, srcs))
+        subprocess.check_call([NVCC, *ARCH, *COMMON, "-o", LIB, *objs])
     return LIB
 
 

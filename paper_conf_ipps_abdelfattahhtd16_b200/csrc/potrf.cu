@@ -44,6 +44,17 @@
 
 namespace vb {
 
+// Every other row block of a panel walks the k chunks backwards (produce_matrix3); 0 disables.
+#ifndef VB_KREV
+#define VB_KREV 1
+#endif
+// SPOTRF's panel update on the FP32 FFMA pipe (k_loop_ffma) instead of FP64 DMMA: a measured
+// experiment, off in the product (C5 FP32 174 ms vs 152 ms with DMMA); build with
+// -DVB_SPOTRF_FFMA=1 to reproduce.
+#ifndef VB_SPOTRF_FFMA
+#define VB_SPOTRF_FFMA 0
+#endif
+
 // Optional phase timers (debug builds with -DVB_PHASE_PROF): warp 0 lane 0 of each CTA of the
 // v2 kernel accumulates clock64() cycles per phase; read with vbatched_debug_phases().
 #ifdef VB_PHASE_PROF
@@ -279,21 +290,24 @@ VB_DEVINL void mm32_quarter(double (&acc)[2][2][2], int wg, int lane, FA fa, FB 
 // aliased with anything, so the producer keeps prefetching across row blocks and panels.
 // E: the matrices' storage type (double for DPOTRF, float for SPOTRF); the ring stages hold E,
 // everything from the fragments on is FP64 (DMMA). Ring leading dims padded so that the
-// fragment loads are bank-conflict free (+4 doubles / +8 floats).
+// DMMA fragment loads are bank-conflict free (+4 doubles / +8 floats); with VB_SPOTRF_FFMA the
+// FP32 stages are read only by the FFMA k-loop, whose lanes all read the same k row (no padding).
 template <int NB_, int KC_, int STAGES_, int MINB_, int WARPS_ = 8, typename E_ = double>
 struct Cfg2 {
   using E = E_;
   static constexpr int NB = NB_, KC = KC_, STAGES = STAGES_, MINB = MINB_;
   static constexpr int WARPS = WARPS_;       // compute warps (16 rows each)
   static constexpr int THREADS = 32 * WARPS, MB = 16 * WARPS, NT = NB / 8;
-  static constexpr int PAD = sizeof(E_) == 8 ? 4 : 8;
+  static constexpr int PAD = sizeof(E_) == 8 ? 4 : (VB_SPOTRF_FFMA ? 0 : 8);
   static constexpr int LDA = MB + PAD, LDB = NB + PAD, LDT = NB + 4;
   static constexpr int G = 16 / (int)sizeof(E_);  // elements per 16 bytes (bulk-copy granule)
 };
 // 3 CTAs/SM: 4 compute warps (MB = NB) + 1 producer; ring of 2 x 16-column chunks (measured
 // against 3 x 8 and 4 x 8: C5 154.4 / 160.5 vs 152.3 ms, the per-chunk barrier cost dominates)
 using Cfg64d = Cfg2<64, 16, 2, 3, 4>;
-using Cfg64s = Cfg2<64, 16, 2, 3, 4, float>;  // the same for FP32 storage (SPOTRF)
+// FP32 storage (SPOTRF). With the FFMA k-loop the unpadded 16-column FP32 chunks leave room for a
+// third ring stage.
+using Cfg64s = Cfg2<64, 16, VB_SPOTRF_FFMA ? 3 : 2, 3, 4, float>;
 
 template <class C>
 struct Smem2 {
@@ -306,6 +320,9 @@ struct Smem2 {
   double wbuf[64];
   double sv[C::NB];
   double tv[C::NB];
+  // VB_SPOTRF_FFMA only: per-warp staging of the FFMA k-loop's FP32 partial sums (one 16 x 32
+  // half of the warp's 16 x 64 tile at a time) on their way into the FP64 fragment layout
+  alignas(16) float xs[(VB_SPOTRF_FFMA && sizeof(typename C::E) == 4) ? C::WARPS : 1][16][40];
   uint64_t full[C::STAGES];
   uint64_t empty[C::STAGES];
   uint64_t panel_done;  // v3: one phase per panel (8 consumer-warp arrivals)
@@ -313,6 +330,9 @@ struct Smem2 {
   int item;
   int info;
 };
+
+static_assert(sizeof(Smem2<Cfg64d>) + 1024 <= 228 * 1024 / 3, "3 CTAs/SM");
+static_assert(sizeof(Smem2<Cfg64s>) + 1024 <= 228 * 1024 / 3, "3 CTAs/SM");
 
 // Diagonal 64x64 block by warps 0..3 (named barrier 1): L11 = potf2(C11), inv(L11) -> T12,
 // L21 = C21 inv(L11)^T -> T21, C22 -= L21 L21^T, L22 = potf2(C22), inv(L22) -> T11.
@@ -587,8 +607,11 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const typename C::E* A, int n, int l
         const int rn = (min(MB, n - r0) + G - 1) / G * G;
         bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + r0, rn * (int)sizeof(E));
       }
-      for (int kc = (r0 == j0 ? nk_free : 0); kc < nk; ++kc)
-        issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, r0, j0, lane, bulk);
+      // Every other row block walks the k chunks backwards, so the panel rows' chunks it reads
+      // first are the ones the previous block read last (still in L2)
+      const bool rev = VB_KREV && (((r0 - j0) / MB) & 1);
+      for (int i = (r0 == j0 ? nk_free : 0); i < nk; ++i)
+        issue_chunk2<C, UP>(s, gchunk++, rev ? nk - 1 - i : i, A, n, ld, r0, j0, lane, bulk);
     }
   }
   gpanel += done;
@@ -628,6 +651,71 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
   }
 }
 
+// VB_SPOTRF_FFMA (FP32 storage): the panel update -= L[r0:, 0:j0] L[j0:j0+64, 0:j0]^T on the FP32
+// FFMA pipe instead of DMMA. Register tile 4 rows x 8 columns per lane
+// (rows wrow + 4 rg .. +3, columns 4 cg .. +3 and 32 + 4 cg .. +3; rg = lane / 8, cg = lane % 8):
+// per k one LDS.128 of A (broadcast) and two LDS.128 of B feed 32 FFMAs. HALF: the columns
+// 32..63 are skipped (a panel's first row block, warps whose rows are all < 32). The FP32 sums
+// join A's values in FP64 in ffma_to_acc; everything after the update stays FP64.
+template <class C, bool HALF>
+VB_DEVINL void k_loop_ffma(Smem2<C>& s, float (&c)[4][8], uint32_t& gchunk, int nk, int wrow,
+                           int lane) {
+  const int rg = lane >> 3, cg = lane & 7;
+  for (int kc = 0; kc < nk; ++kc) {
+    const uint32_t gi = gchunk++;
+    const int st = gi % C::STAGES;
+    mbar_wait(&s.full[st], (gi / C::STAGES) & 1);
+#pragma unroll
+    for (int k = 0; k < C::KC; ++k) {
+      const float4 a = *reinterpret_cast<const float4*>(&s.a[st][k][wrow + rg * 4]);
+      const float4 b0 = *reinterpret_cast<const float4*>(&s.b[st][k][cg * 4]);
+      const float av[4] = {a.x, a.y, a.z, a.w};
+      float bv[8] = {b0.x, b0.y, b0.z, b0.w, 0.f, 0.f, 0.f, 0.f};
+      if (!HALF) {
+        const float4 b1 = *reinterpret_cast<const float4*>(&s.b[st][k][32 + cg * 4]);
+        bv[4] = b1.x;
+        bv[5] = b1.y;
+        bv[6] = b1.z;
+        bv[7] = b1.w;
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < (HALF ? 4 : 8); ++j) c[i][j] = fmaf(-av[i], bv[j], c[i][j]);
+    }
+    fence_proxy_async();  // see k_loop3
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&s.empty[st]);
+  }
+}
+
+// acc (FP64 fragment layout) = A's values a0 + the FFMA tile c, through the warp's xs staging in
+// two 32-column halves (STS.128 per lane row, LDS.64 in the fragment layout; row stride 40 floats
+// keeps each half-warp on 32 distinct banks).
+template <class C>
+VB_DEVINL void ffma_to_acc(Smem2<C>& s, const float (&c)[4][8], const float (&a0)[2][C::NT][2],
+                           double (&acc)[2][C::NT][2], int warp, int lane) {
+  const int rg = lane >> 3, cg = lane & 7, g = lane >> 2, q = lane & 3;
+  float(*x)[40] = s.xs[warp];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      *reinterpret_cast<float4*>(&x[rg * 4 + i][cg * 4]) =
+          make_float4(c[i][4 * h], c[i][4 * h + 1], c[i][4 * h + 2], c[i][4 * h + 3]);
+    __syncwarp();
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < 4; ++nt) {
+        const float2 v = *reinterpret_cast<const float2*>(&x[mt * 8 + g][nt * 8 + 2 * q]);
+        acc[mt][4 * h + nt][0] = (double)a0[mt][4 * h + nt][0] + (double)v.x;
+        acc[mt][4 * h + nt][1] = (double)a0[mt][4 * h + nt][1] + (double)v.y;
+      }
+    __syncwarp();
+  }
+}
+
 template <class C, bool UP>
 VB_DEVINL void consume_matrix3(Smem2<C>& s, typename C::E* __restrict__ A, int n, int ld,
                                int* info_out, uint32_t& gchunk, uint32_t& gpanel) {
@@ -653,7 +741,11 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, typename C::E* __restrict__ A, int n
         }
         continue;
       }
-      double acc[2][NT][2];
+      // A's panel values in the storage type (FP32 for SPOTRF), entries outside the panel's
+      // lower part 0
+      using E = typename C::E;
+      constexpr bool kFfma = VB_SPOTRF_FFMA && sizeof(E) == 4;
+      E a0[2][NT][2];
 #pragma unroll
       for (int mt = 0; mt < 2; ++mt)
 #pragma unroll
@@ -662,14 +754,51 @@ VB_DEVINL void consume_matrix3(Smem2<C>& s, typename C::E* __restrict__ A, int n
           for (int h = 0; h < 2; ++h) {
             const int row = r0 + wrow + mt * 8 + g, col = j0 + nt * 8 + 2 * q + h;
             const bool v = row < n && col < j0 + nb && row >= col;
-            acc[mt][nt][h] = v ? __ldcg(A + gix<UP>(row, col, ld)) : 0.0;
+            a0[mt][nt][h] = v ? __ldcg(A + gix<UP>(row, col, ld)) : E(0);
           }
+      double acc[2][NT][2];
+      if constexpr (!kFfma) {
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) acc[mt][nt][h] = a0[mt][nt][h];
+      }
       VB_T0(t_k)
       // In a panel's first row block the diagonal-block warps only need the column tiles on
       // or below their rows (SYRK): compile-time variants skip the strictly upper tiles.
       const int ntl = (first && wrow < NB) ? (wrow + 16) / 8 : NT;
       if (!active) {
         k_loop3<C, 0>(s, acc, gchunk, nk, wrow, lane);
+        if constexpr (kFfma) {
+#pragma unroll
+          for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+              for (int h = 0; h < 2; ++h) acc[mt][nt][h] = a0[mt][nt][h];
+        }
+      } else if constexpr (kFfma) {
+        float c[4][8];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) c[i][j] = 0.f;
+        if (ntl <= 4)
+          k_loop_ffma<C, true>(s, c, gchunk, nk, wrow, lane);
+        else
+          k_loop_ffma<C, false>(s, c, gchunk, nk, wrow, lane);
+        // entries outside the panel's lower part (stale ring rows/columns included) are dropped
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const int row = r0 + wrow + (lane >> 3) * 4 + i;
+            const int col = j0 + (j < 4 ? 0 : 32) + (lane & 7) * 4 + (j & 3);
+            c[i][j] = (row < n && col < j0 + nb && row >= col) ? c[i][j] : 0.f;
+          }
+        ffma_to_acc<C>(s, c, a0, acc, warp, lane);
       } else if (ntl == 2) {
         k_loop3<C, 2>(s, acc, gchunk, nk, wrow, lane);
       } else if (ntl == 4) {

@@ -85,6 +85,41 @@ __global__ void __launch_bounds__(128, 4) dmma_tile(double* out, int iters) {
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
+// The SPOTRF blocked kernel's FFMA shape (potrf.cu k_loop_ffma): warp w owns rows 16w..16w+15 x
+// 64 columns, lane (rg, cg) rows 16w + 4 rg .. +3, columns 4 cg .. +3 and 32 + 4 cg .. +3.
+// MAP 0: rg = lane / 8, cg = lane % 8; MAP 1: rg = lane % 4, cg = lane / 4.
+template <int MAP>
+__global__ void __launch_bounds__(128) ffma_tile16(float* out, int iters) {
+  __shared__ __align__(16) float A[16][64], B[16][64];
+  for (int e = threadIdx.x; e < 16 * 64; e += 128) {
+    A[e / 64][e % 64] = 1e-3f * (e % 7);
+    B[e / 64][e % 64] = 1e-3f * (e % 5);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int rg = MAP ? (lane & 3) : (lane >> 3), cg = MAP ? (lane >> 2) : (lane & 7);
+  const int r0 = warp * 16 + rg * 4;
+  float acc[4][8] = {};
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int k = 0; k < 16; ++k) {
+      const float4 a = *reinterpret_cast<const float4*>(&A[k][r0]);
+      const float4 b0 = *reinterpret_cast<const float4*>(&B[k][cg * 4]);
+      const float4 b1 = *reinterpret_cast<const float4*>(&B[k][32 + cg * 4]);
+      const float av[4] = {a.x, a.y, a.z, a.w};
+      const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(-av[i], bv[j], acc[i][j]);
+    }
+  }
+  float s = 0;
+  for (int i = 0; i < 4; ++i)
+    for (int j = 0; j < 8; ++j) s += acc[i][j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 int main() {
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
@@ -112,6 +147,13 @@ int main() {
       [&] { ffma_peak<<<grid, 128>>>(fo, it1); }, 2.0 * grid * 128 * 8 * (double)it1);
   run("ffma_tile (64x64 tile, 4x8 per thread, LDS.128 operands)",
       [&] { ffma_tile<<<grid, 128>>>(fo, it2); }, 2.0 * grid * 64.0 * 64 * 64 * it2);
+  for (int cps = 3; cps <= 4; ++cps) {
+    char nm[160];
+    snprintf(nm, sizeof nm, "ffma_tile16 MAP0 (SPOTRF kernel shape, 16x64 per warp, %d CTAs/SM)", cps);
+    run(nm, [&] { ffma_tile16<0><<<sms * cps, 128>>>(fo, it2 * 4); }, 2.0 * sms * cps * 64.0 * 64 * 16 * it2 * 4);
+    snprintf(nm, sizeof nm, "ffma_tile16 MAP1 (SPOTRF kernel shape, 16x64 per warp, %d CTAs/SM)", cps);
+    run(nm, [&] { ffma_tile16<1><<<sms * cps, 128>>>(fo, it2 * 4); }, 2.0 * sms * cps * 64.0 * 64 * 16 * it2 * 4);
+  }
   run("dmma_tile (blocked-kernel k-loop shape, 16x64 per warp)",
       [&] { dmma_tile<<<grid, 128>>>(dout, it3); }, 2.0 * grid * 64.0 * 64 * 16 * it3);
   printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));

@@ -24,7 +24,7 @@ else:
     seed = vbgen.CONFIGS[cfg].seed
 if lim:
     n = n[:lim]
-db = DeviceBatch(n, seed=seed).fill()
+db = DeviceBatch(n, seed=seed, dtype=os.environ.get("DTYPE", "f64")).fill()
 L = vb.lib()
 L.vbatched_debug_phases.argtypes = [ctypes.c_void_p, ctypes.c_int]
 out = (ctypes.c_ulonglong * 8)()
@@ -50,7 +50,7 @@ if os.environ.get("QUAD"):  # quad small kernel: slots 0-2 chain warp, 3-6 the 3
         print(f"  {nm:18s} {v:16.0f}  {100.0 * v / max(tot, 1):6.1f} % of matrix time")
     sys.exit(0)
 names = (["gemm", "potf2", "trtri", "trsm", "matrix_total", "panel_bar"] if os.environ.get("SMALL") else
-         ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "acc_init"])
+         ["kloop", "diag", "trsm+store", "panel_end", "matrix_total", "kloop_full_wait"])
 tot = out[4]
 print(f"{cfg} lim={lim} kernel {e0.elapsed_time(e1):.3f} ms; per-CTA-warp0 cycles (sum over CTAs):")
 for i, nm in enumerate(names):
