@@ -97,14 +97,46 @@ __global__ void __launch_bounds__(1024, 1) tile_scan_kernel(BlasArgs a, int* off
   }
 }
 
-__device__ __forceinline__ int find_matrix(const int* off, int batch, int t) {
-  int lo = 0, hi = batch;  // largest i with off[i] <= t and tiles > 0
+// Tile -> matrix lookup (the matrix of tile t is the largest i with off[i] <= t; it has tiles,
+// since off[i+1] > t). A binary search over off[] in global memory is a chain of ~log2(batch)
+// dependent L2 round trips per tile (12 for 3000 matrices, several microseconds), which
+// dominated the tiny rank-16 tiles of GETRF/GEQRF's trailing updates. Instead every CTA samples
+// off[] once (coarse[c] = off[c S], S a multiple of 32 with at most kCoarse samples), and a tile
+// is located by a binary search in shared memory plus one round of S / 32 independent
+// coalesced warp loads of off[] and a ballot.
+constexpr int kCoarse = 512;
+struct TileIndex {
+  int coarse[kCoarse];
+  int S, nc;
+};
+
+__device__ __forceinline__ void tile_index_init(TileIndex& x, const int* off, int batch) {
+  const int S = max(32, cdiv(cdiv(batch, kCoarse), 32) * 32);
+  const int nc = cdiv(batch, S);
+  for (int c = threadIdx.x; c < nc; c += blockDim.x) x.coarse[c] = off[c * S];
+  if (threadIdx.x == 0) {
+    x.S = S;
+    x.nc = nc;
+  }
+  __syncthreads();
+}
+
+// One warp (all lanes get the result).
+__device__ __forceinline__ int tile_locate(const TileIndex& x, const int* off, int batch, int t,
+                                           int lane) {
+  int lo = 0, hi = x.nc;
   while (hi - lo > 1) {
     const int mid = (lo + hi) >> 1;
-    if (off[mid] <= t) lo = mid;
+    if (x.coarse[mid] <= t) lo = mid;
     else hi = mid;
   }
-  return lo;
+  const int base = lo * x.S;
+  int cnt = 0;
+  for (int u = 0; u < x.S; u += 32) {
+    const int i = base + u + lane;
+    cnt += __popc(__ballot_sync(kFull, i < batch && off[i] <= t));
+  }
+  return base + cnt - 1;
 }
 
 // ---------------------------------------------------------------------------------------
@@ -145,19 +177,30 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
                                                                  int* counter) {
   extern __shared__ __align__(16) unsigned char gsm_raw[];
   GemmSmem& s = *reinterpret_cast<GemmSmem*>(gsm_raw);
-  __shared__ int s_t;
+  __shared__ int s_t, s_mi;
+  __shared__ TileIndex tix;
   pdl_wait();
   const int total = off[a.batch];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int g = lane >> 2, q = lane & 3;
   const int wr = (warp >> 1) * 32, wc = (warp & 1) * 32;
+  tile_index_init(tix, off, a.batch);
+  // the next tile id is popped while the current tile runs (thread 0 stores it at the loop top)
+  int nxt = 0;
+  if (tid == 0) nxt = atomicAdd(counter, 1);
   for (;;) {
-    if (tid == 0) s_t = atomicAdd(counter, 1);
+    if (tid == 0) s_t = nxt;
+    __syncthreads();
+    if (warp == 0) {
+      const int tt = s_t;
+      const int mm = tt < total ? tile_locate(tix, off, a.batch, tt, lane) : 0;
+      if (lane == 0) s_mi = mm;
+    }
     __syncthreads();
     const int t = s_t;
-    __syncthreads();
     if (t >= total) break;
-    const int mi = find_matrix(off, a.batch, t);
+    if (tid == 0) nxt = atomicAdd(counter, 1);
+    const int mi = s_mi;
     int lt = t - off[mi];
     const int n = a.n[mi];
     const int m = (a.mode == kGemm) ? a.m[mi] : n;
@@ -326,19 +369,29 @@ __device__ __forceinline__ void trsm_stage(TrsmSmem& s, int st, const BlasArgs& 
 __global__ void __launch_bounds__(kGThreads) trsm_kernel(BlasArgs a, const int* off, int* counter) {
   extern __shared__ __align__(16) unsigned char tsm_raw[];
   TrsmSmem& s = *reinterpret_cast<TrsmSmem*>(tsm_raw);
-  __shared__ int s_t;
+  __shared__ int s_t, s_mi;
+  __shared__ TileIndex tix;
   pdl_wait();
   const int total = off[a.batch];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int g = lane >> 2, q = lane & 3;
   const int wr = (warp >> 1) * 32, wc = (warp & 1) * 16;
+  tile_index_init(tix, off, a.batch);
+  int nxt = 0;  // the next tile id, popped while the current one runs (see gemm_syrk_kernel)
+  if (tid == 0) nxt = atomicAdd(counter, 1);
   for (;;) {
-    if (tid == 0) s_t = atomicAdd(counter, 1);
+    if (tid == 0) s_t = nxt;
+    __syncthreads();
+    if (warp == 0) {
+      const int tt = s_t;
+      const int mm = tt < total ? tile_locate(tix, off, a.batch, tt, lane) : 0;
+      if (lane == 0) s_mi = mm;
+    }
     __syncthreads();
     const int t = s_t;
-    __syncthreads();
     if (t >= total) break;
-    const int mi = find_matrix(off, a.batch, t);
+    if (tid == 0) nxt = atomicAdd(counter, 1);
+    const int mi = s_mi;
     const int r0 = (t - off[mi]) * kBT;
     const int m = a.m[mi], n = a.n[mi];
     const double* A = a.A[mi];
