@@ -234,9 +234,26 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
 #pragma unroll
       for (int y = 0; y < 4; ++y) acc[x][y][0] = acc[x][y][1] = 0.0;
     const int nk = cdiv(K, kBK);
+    double* C = a.C[mi];
+    const int ldc = a.ldc[mi];
+    // One k chunk (K <= 16: the rank-16 trailing updates of GETRF/GEQRF): the C tile is fetched
+    // into the idle ring stages 1-2 together with the chunk, so its load latency overlaps the
+    // chunk's instead of following the products (columns 0..31 in a[1..2], 32..63 in b[1..2]).
+    const bool cpre = nk == 1 && a.beta != 0.0;
+    auto cs = [&](int c, int r) -> double* {
+      return (c < 32 ? &s.a[1][0][0] : &s.b[1][0][0]) + (c & 31) * kLD + r;
+    };
     if (nk > 0) gemm_stage(s, 0, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, 0);
     cp_async_commit();
     if (nk > 1) gemm_stage(s, 1, A, lda, a.ta, B, ldb, a.tb, m, n, K, r0, c0, kBK);
+    if (cpre) {
+#pragma unroll 4
+      for (int e = tid; e < kBT * kBT; e += kGThreads) {
+        const int r = e % kBT, c = e / kBT;
+        const bool p = r0 + r < m && c0 + c < n;
+        cp_async8(cs(c, r), C + (p ? (size_t)(c0 + c) * ldc + (r0 + r) : 0), p);
+      }
+    }
     cp_async_commit();
     for (int kc = 0; kc < nk; ++kc) {
       cp_async_wait<1>();  // chunk kc has landed (only chunk kc+1 may still be in flight)
@@ -260,9 +277,8 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
       }
     }
     cp_async_wait<0>();
-    __syncthreads();  // the next tile's prologue refills stages 0 and 1
-    double* C = a.C[mi];
-    const int ldc = a.ldc[mi];
+    __syncthreads();  // the C tile has landed (cpre); the next tile's prologue refills stages 0-1
+                      // only after the loop-top barriers, when every thread has read it
     // Epilogue in two passes: every load of C first (all in flight together), then every store.
     // As one read-modify-write per element the loads serialise behind the stores (the compiler
     // cannot move a load of C past a store to C): one memory round trip per element, most of a
@@ -277,7 +293,8 @@ __global__ void __launch_bounds__(kGThreads, 4) gemm_syrk_kernel(BlasArgs a, con
             const int r = r0 + wr + x * 8 + g, c = c0 + wc + y * 8 + 2 * q + h;
             const bool p = r < m && c < n && !(a.mode == kSyrkLower && r < c) &&
                            !(a.mode == kSyrkUpper && r > c);
-            acc[x][y][h] = a.alpha * acc[x][y][h] + (p ? a.beta * C[(size_t)c * ldc + r] : 0.0);
+            const double cv = !p ? 0.0 : cpre ? *cs(c - c0, r - r0) : C[(size_t)c * ldc + r];
+            acc[x][y][h] = a.alpha * acc[x][y][h] + (p ? a.beta * cv : 0.0);
           }
     } else {
 #pragma unroll
