@@ -7,12 +7,19 @@
 // Built the paper's "separated" way: a host loop over panels of NB columns,
 // each step = an aux kernel that derives the per-matrix sub-problem sizes and pointers on the
 // GPU (the size arrays live there), a fused panel kernel (getf2 with partial
-// pivoting, rows in registers), the row interchanges on the columns right of the panel fused
-// with the unit-lower solve A12 <- L11^-1 A12 (laswp + trsm, one warp per column), and then the
-// SAME vbatched GEMM kernel that vbatched_dgemm exports:
-//   A22 <- A22 - A21 A12 (vbatched GEMM, DMMA)
-// The interchanges on the columns left of each panel are applied once after the last step.
-// Matrices whose panel is exhausted get size 0 in the step arrays and cost no tiles.
+// pivoting, rows in registers), the row interchanges fused with the unit-lower solve
+// A12 <- L11^-1 A12 (laswp + trsm, one warp per column), and then the SAME vbatched GEMM and
+// TRSM kernels that vbatched_dgemm / vbatched_dtrsm export, in two levels, so that the trailing
+// matrix is streamed once per 64 columns instead of once per 16 (rank-16 updates are HBM-bound):
+//   inner step j (16 columns of the 64-column block [j0, j0 + 64), restricted to the block):
+//     panel j; interchanges on the block's other columns; solve of rows j..j+15 of the block's
+//     columns right of the panel; A[j+16:, j+16:j0+64] -= A21 A12 (vbatched GEMM, k = 16)
+//   after the block (LAPACK DGETRF's blocked step, the block playing the panel):
+//     the block's interchanges on the trailing columns (lu_laswp_block_kernel);
+//     A[j0:j0+64, j0+64:] <- L11^-1 A[j0:j0+64, j0+64:] (vbatched DTRSM, unit lower 64 x 64);
+//     A[j0+64:, j0+64:] -= A[j0+64:, j0:j0+64] A[j0:j0+64, j0+64:] (vbatched GEMM, k = 64).
+// The interchanges of later blocks reach the columns of earlier blocks once, after the last
+// step. Matrices whose panel is exhausted get size 0 in the step arrays and cost no tiles.
 #include <algorithm>
 
 #include "../../include/vbatched.h"
@@ -22,19 +29,25 @@
 namespace vb {
 namespace {
 
-constexpr int kLuNB = 16;        // panel width (the trailing GEMM's k)
+constexpr int kLuNB = 16;        // panel width (the inner GEMMs' k)
+constexpr int kLuOB = 64;        // outer block width (the trailing GEMM's k)
 constexpr int kLuThreads = 256;  // panel kernel CTA
 constexpr int kLuMaxRPT = 4;     // rows per thread held in registers: m - j <= 1024
 
 struct LuStep {
   int* pm;   // panel rows (m_i - j), 0 when the matrix has no panel at step j
   int* pn;   // panel width (<= NB)
-  int* rn;   // columns right of the panel
-  int* bm;   // rows below the panel
-  double** P;    // panel top-left A_i(j, j)
-  double** A12;  // A_i(j, j + pn)
-  double** A21;  // A_i(j + pn, j)
-  double** A22;  // A_i(j + pn, j + pn)
+  double** P;  // panel top-left A_i(j, j)
+  // BLAS problems, 2 x batch entries: inner step [0, batch) the GEMM in the block; after a
+  // block [0, batch) the k = 64 trailing GEMM and [batch, 2 batch) the TRSM (gm x gn right-hand
+  // side at gB, unit lower gA)
+  int* gm;
+  int* gn;
+  int* gk;
+  int* gld;  // ldda_i, twice
+  double** gA;
+  double** gB;
+  double** gC;
 };
 
 // info: -1 m < 0, -2 n < 0, -4 ldda < max(1, m), -9 m > max_m or n > max_n; else 0.
@@ -54,21 +67,52 @@ __global__ void lu_validate_kernel(const int* __restrict__ d_m, const int* __res
 
 __global__ void lu_step_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
                                double* const* __restrict__ dA, const int* __restrict__ d_ld,
-                               const int* __restrict__ d_info, int batch, int j, LuStep st) {
+                               const int* __restrict__ d_info, int batch, int j, int j0, LuStep st) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
     const int m = d_m[i], n = d_n[i], ld = d_ld[i];
     const int kmax = m < n ? m : n;
     const bool act = d_info[i] >= 0 && j < kmax;
     const int nb = act ? min(kLuNB, kmax - j) : 0;
+    const int oend = min(j0 + kLuOB, n);  // the block's last column + 1
     st.pm[i] = act ? m - j : 0;
     st.pn[i] = nb;
-    st.rn[i] = act ? n - j - nb : 0;
-    st.bm[i] = act ? m - j - nb : 0;
     double* A = dA[i];
     st.P[i] = act ? A + (size_t)j * ld + j : A;
-    st.A12[i] = act ? A + (size_t)(j + nb) * ld + j : A;
-    st.A21[i] = act ? A + (size_t)j * ld + j + nb : A;
-    st.A22[i] = act ? A + (size_t)(j + nb) * ld + j + nb : A;
+    const int r1 = j + nb;  // first row / column after the panel
+    st.gld[i] = st.gld[batch + i] = ld;
+    st.gk[i] = nb;
+    st.gA[i] = act ? A + (size_t)j * ld + r1 : A;  // L21
+    // the block's columns right of the panel, all rows below
+    st.gm[i] = act ? m - r1 : 0;
+    st.gn[i] = act ? max(0, oend - r1) : 0;
+    st.gB[i] = act ? A + (size_t)r1 * ld + j : A;
+    st.gC[i] = act ? A + (size_t)r1 * ld + r1 : A;
+  }
+}
+
+// After the block [j0, j0 + 64): the TRSM of the block's rows of the trailing columns with the
+// block's unit lower L11 (entries [batch, 2 batch)), and the k = 64 GEMM below (entries [0, batch)).
+__global__ void lu_block_step_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                                     double* const* __restrict__ dA, const int* __restrict__ d_ld,
+                                     const int* __restrict__ d_info, int batch, int j0, LuStep st) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    const int kmax = m < n ? m : n;
+    const int e = j0 + kLuOB;
+    const int kb = min(kLuOB, kmax - j0);  // the block's panel columns
+    const bool tr = d_info[i] >= 0 && kb > 0 && e < n;      // trailing columns exist
+    const bool gm = tr && e < m;                            // and rows below the block
+    double* A = dA[i];
+    st.gm[batch + i] = tr ? kb : 0;
+    st.gn[batch + i] = tr ? n - e : 0;
+    st.gA[batch + i] = tr ? A + (size_t)j0 * ld + j0 : A;
+    st.gB[batch + i] = tr ? A + (size_t)e * ld + j0 : A;
+    st.gm[i] = gm ? m - e : 0;
+    st.gn[i] = gm ? n - e : 0;
+    st.gk[i] = gm ? kLuOB : 0;
+    st.gA[i] = gm ? A + (size_t)j0 * ld + e : A;
+    st.gB[i] = gm ? A + (size_t)e * ld + j0 : A;
+    st.gC[i] = gm ? A + (size_t)e * ld + e : A;
   }
 }
 
@@ -234,7 +278,7 @@ __device__ int lu_step_perm(const int* ip, int j, int pn, int* srow, int* ssrc) 
 __global__ void __launch_bounds__(256)
     lu_laswp_trsm_kernel(LuStep st, double* const* __restrict__ dA, const int* __restrict__ d_n,
                          const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv, int batch,
-                         int j) {
+                         int j, int j0) {
   __shared__ int srow[2 * kLuNB];  // S
   __shared__ int ssrc[2 * kLuNB];  // for slot t: the slot whose old value moves to S[t]
   __shared__ int s_cnt;
@@ -243,7 +287,8 @@ __global__ void __launch_bounds__(256)
     const int pn = st.pn[i];
     if (pn <= 0) continue;
     const int n = d_n[i], ld = d_ld[i];
-    if (j + pn >= n) continue;
+    const int cend = min(j0 + kLuOB, n);  // the block's columns only
+    if (j + pn >= cend && j == j0) continue;
     double* A = dA[i];
     if (threadIdx.x == 0) s_cnt = lu_step_perm(d_ipiv[i] + j, j, pn, srow, ssrc);
     __syncthreads();
@@ -254,7 +299,7 @@ __global__ void __launch_bounds__(256)
     double l11[kLuNB];
 #pragma unroll
     for (int k = 0; k < kLuNB; ++k) l11[k] = (k < lane && lane < pn) ? L11[(size_t)k * ld + lane] : 0.0;
-    for (int c = j + pn + warp; c < n; c += nw) {
+    for (int c = j + pn + warp; c < cend; c += nw) {
       double* col = A + (size_t)c * ld;
       const double v_lo = lane < cnt ? col[r_lo] : 0.0;
       const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
@@ -268,6 +313,55 @@ __global__ void __launch_bounds__(256)
       }
       if (lane < cnt) col[r_lo] = x;
       if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
+    }
+    // the block's columns left of the panel: the interchanges only
+    for (int c = j0 + warp; c < j; c += nw) {
+      double* col = A + (size_t)c * ld;
+      const double v_lo = lane < cnt ? col[r_lo] : 0.0;
+      const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
+      const double a_lo = __shfl_sync(kFull, v_lo, f_lo & 31), b_lo = __shfl_sync(kFull, v_hi, f_lo & 31);
+      const double a_hi = __shfl_sync(kFull, v_lo, f_hi & 31), b_hi = __shfl_sync(kFull, v_hi, f_hi & 31);
+      if (lane < cnt) col[r_lo] = f_lo < 32 ? a_lo : b_lo;
+      if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
+    }
+    __syncthreads();
+  }
+}
+
+// After a block: its steps' interchanges, in order, on the trailing columns (pure data movement;
+// one warp per column moves only the rows of each step's set S).
+__global__ void __launch_bounds__(256)
+    lu_laswp_block_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                          double* const* __restrict__ dA, const int* __restrict__ d_ld,
+                          int* const* __restrict__ d_ipiv, const int* __restrict__ d_info, int batch,
+                          int j0) {
+  __shared__ int srow[2 * kLuNB], ssrc[2 * kLuNB];
+  __shared__ int s_cnt;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (int i = blockIdx.x; i < batch; i += gridDim.x) {
+    if (d_info[i] < 0) continue;
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    const int kmax = m < n ? m : n;
+    const int cbeg = j0 + kLuOB;
+    if (cbeg >= n || j0 >= kmax) continue;
+    double* A = dA[i];
+    for (int j = j0; j < min(cbeg, kmax); j += kLuNB) {
+      const int pn = min(kLuNB, kmax - j);
+      __syncthreads();  // the previous step's columns are done with srow / ssrc
+      if (threadIdx.x == 0) s_cnt = lu_step_perm(d_ipiv[i] + j, j, pn, srow, ssrc);
+      __syncthreads();
+      const int cnt = s_cnt;
+      const int r_lo = lane < cnt ? srow[lane] : 0, r_hi = lane + 32 < cnt ? srow[lane + 32] : 0;
+      const int f_lo = lane < cnt ? ssrc[lane] : 0, f_hi = lane + 32 < cnt ? ssrc[lane + 32] : 0;
+      for (int c = cbeg + warp; c < n; c += nw) {
+        double* col = A + (size_t)c * ld;
+        const double v_lo = lane < cnt ? col[r_lo] : 0.0;
+        const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
+        const double a_lo = __shfl_sync(kFull, v_lo, f_lo & 31), b_lo = __shfl_sync(kFull, v_hi, f_lo & 31);
+        const double a_hi = __shfl_sync(kFull, v_lo, f_hi & 31), b_hi = __shfl_sync(kFull, v_hi, f_hi & 31);
+        if (lane < cnt) col[r_lo] = f_lo < 32 ? a_lo : b_lo;
+        if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
+      }
     }
     __syncthreads();
   }
@@ -297,20 +391,30 @@ __global__ void __launch_bounds__(256)
     double* A = dA[i];
     const int* ip = d_ipiv[i];
     for (int r = tid; r < m; r += blockDim.x) src[r] = r;
-    for (int b = nblk - 2; b >= 0; --b) {
-      const int j = (b + 1) * kLuNB, pn = min(kLuNB, kmax - j);
-      __syncthreads();  // src complete, previous block's buf reads done
-      if (tid == 0) s_cnt = lu_step_perm(ip + j, j, pn, srow, ssrc);
-      __syncthreads();
-      const int cnt = s_cnt;
-      for (int r = j + tid; r < m; r += blockDim.x) {
-        const int x = src[r];
-        int y = x;
-        for (int t = 0; t < cnt; ++t)
-          if (srow[t] == x) y = srow[ssrc[t]];
-        src[r] = y;
+    constexpr int SPB = kLuOB / kLuNB;  // steps per 64-column block
+    int folded = nblk;                  // steps >= folded are in src
+    for (int b = nblk - 1; b >= 0; --b) {
+      // the block of step b received the interchanges of its own block's steps at once
+      // (lu_laswp_trsm_kernel); it still needs those of every later block
+      const int target = (b / SPB + 1) * SPB;
+      while (folded > target) {
+        --folded;
+        const int j = folded * kLuNB, pn = min(kLuNB, kmax - j);
+        __syncthreads();  // src complete, previous block's buf reads done
+        if (tid == 0) s_cnt = lu_step_perm(ip + j, j, pn, srow, ssrc);
+        __syncthreads();
+        const int cnt = s_cnt;
+        for (int r = j + tid; r < m; r += blockDim.x) {
+          const int x = src[r];
+          int y = x;
+          for (int t = 0; t < cnt; ++t)
+            if (srow[t] == x) y = srow[ssrc[t]];
+          src[r] = y;
+        }
       }
-      for (int c = b * kLuNB; c < j; ++c) {
+      if (folded == nblk) continue;  // nothing later
+      const int j = folded * kLuNB;   // rows >= j may move
+      for (int c = b * kLuNB; c < min((b + 1) * kLuNB, kmax); ++c) {
         double* col = A + (size_t)c * ld;
         __syncthreads();  // src updated; buf free
         for (int r = j + tid; r < m; r += blockDim.x) buf[r] = col[r];
@@ -342,40 +446,58 @@ int getrf_impl(const int* d_m, const int* d_n, double* const* dA, const int* d_l
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   void* ws = nullptr;
   const size_t ibytes = sizeof(int) * (size_t)batch, pbytes = sizeof(double*) * (size_t)batch;
-  cudaError_t e = ws_alloc(&ws, 4 * ibytes + 4 * pbytes + 64, stream);
+  cudaError_t e = ws_alloc(&ws, 2 * ibytes + pbytes + 8 * ibytes + 6 * pbytes + 64, stream);
   if (e != cudaSuccess) return (int)e;
   char* w = static_cast<char*>(ws);
   LuStep st;
   st.P = reinterpret_cast<double**>(w);
-  st.A12 = st.P + batch;
-  st.A21 = st.A12 + batch;
-  st.A22 = st.A21 + batch;
-  st.pm = reinterpret_cast<int*>(st.A22 + batch);
+  st.gA = st.P + batch;
+  st.gB = st.gA + 2 * batch;
+  st.gC = st.gB + 2 * batch;
+  st.pm = reinterpret_cast<int*>(st.gC + 2 * batch);
   st.pn = st.pm + batch;
-  st.rn = st.pn + batch;
-  st.bm = st.rn + batch;
+  st.gm = st.pn + batch;
+  st.gn = st.gm + 2 * batch;
+  st.gk = st.gn + 2 * batch;
+  st.gld = st.gk + 2 * batch;
   const int eg = std::max(1, std::min((batch + 255) / 256, 4 * sms));
   lu_validate_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, d_ld, d_info, batch, max_m, max_n);
   e = cudaGetLastError();
   const int kmax = std::min(max_m, max_n);
   const int pg = std::max(1, std::min(batch, 8 * sms));
-  for (int j = 0; j < kmax && e == cudaSuccess; j += kLuNB) {
-    lu_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, batch, j, st);
-    if ((e = cudaGetLastError()) != cudaSuccess) break;
-    const int rows = max_m - j;
-    if (rows <= kLuThreads) e = launch_panel<1>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
-    else if (rows <= 2 * kLuThreads) e = launch_panel<2>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
-    else e = launch_panel<4>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
-    if (e != cudaSuccess) break;
-    if (j + kLuNB < max_n) {
-      lu_laswp_trsm_kernel<<<pg, 256, 0, stream>>>(st, dA, d_n, d_ld, d_ipiv, batch, j);
+  for (int j0 = 0; j0 < kmax && e == cudaSuccess; j0 += kLuOB) {
+    for (int j = j0; j < std::min(j0 + kLuOB, kmax) && e == cudaSuccess; j += kLuNB) {
+      lu_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, batch, j, j0, st);
       if ((e = cudaGetLastError()) != cudaSuccess) break;
-      int rc = gemm_launch('N', 'N', st.bm, st.rn, st.pn, -1.0, st.A21, d_ld, st.A12, d_ld, 1.0,
-                           st.A22, d_ld, batch, max_m, max_n, kLuNB, stream);
-      if (rc != 0) {
-        e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
-        break;
+      const int rows = max_m - j;
+      if (rows <= kLuThreads) e = launch_panel<1>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+      else if (rows <= 2 * kLuThreads) e = launch_panel<2>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+      else e = launch_panel<4>(pg, st, d_ld, d_ipiv, d_info, batch, j, stream);
+      if (e != cudaSuccess) break;
+      if (j + kLuNB < std::min(j0 + kLuOB, max_n) || j > j0) {
+        lu_laswp_trsm_kernel<<<pg, 256, 0, stream>>>(st, dA, d_n, d_ld, d_ipiv, batch, j, j0);
+        if ((e = cudaGetLastError()) != cudaSuccess) break;
       }
+      if (j + kLuNB < std::min(j0 + kLuOB, max_n)) {
+        int rc = gemm_launch('N', 'N', st.gm, st.gn, st.gk, -1.0, st.gA, st.gld, st.gB, st.gld, 1.0,
+                             st.gC, st.gld, batch, max_m, max_n, kLuNB, stream);
+        if (rc != 0) {
+          e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
+          break;
+        }
+      }
+    }
+    if (e == cudaSuccess && j0 + kLuOB < max_n) {
+      lu_laswp_block_kernel<<<pg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_ipiv, d_info, batch, j0);
+      if ((e = cudaGetLastError()) != cudaSuccess) break;
+      lu_block_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, batch, j0, st);
+      if ((e = cudaGetLastError()) != cudaSuccess) break;
+      int rc = trsm_launch('L', 'L', 'N', 'U', st.gm + batch, st.gn + batch, 1.0, st.gA + batch,
+                           st.gld, st.gB + batch, st.gld, batch, kLuOB, max_n, stream);
+      if (rc == 0 && j0 + kLuOB < max_m)
+        rc = gemm_launch('N', 'N', st.gm, st.gn, st.gk, -1.0, st.gA, st.gld, st.gB, st.gld, 1.0,
+                         st.gC, st.gld, batch, max_m, max_n, kLuOB, stream);
+      if (rc != 0) e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
     }
   }
   if (e == cudaSuccess && kmax > kLuNB) {
