@@ -242,9 +242,10 @@ __global__ void __launch_bounds__(kLuThreads)
 // only moves rows of the set S = {j..j+pn-1} u {ipiv targets} (<= 2 pn <= 64 rows): a
 // permutation of S, built by one thread. Slot t holds row srow[t]; after the interchanges row
 // srow[t] holds the old value of row srow[ssrc[t]]. Slots 0..pn-1 are rows j..j+pn-1.
+template <int CAP = 2 * kLuNB>
 __device__ int lu_step_perm(const int* ip, int j, int pn, int* srow, int* ssrc) {
   int cnt = pn;
-  int cur[2 * kLuNB];  // cur[t]: slot whose original value currently sits in S[t]
+  int cur[CAP];  // cur[t]: slot whose original value currently sits in S[t]
   for (int t = 0; t < pn; ++t) {
     srow[t] = j + t;
     cur[t] = t;
@@ -328,14 +329,18 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-// After a block: its steps' interchanges, in order, on the trailing columns (pure data movement;
-// one warp per column moves only the rows of each step's set S).
+// After a block: its interchanges on the trailing columns (pure data movement). The block's kb
+// pivots are composed into one permutation of the rows they touch (rows j0..j0+kb-1 plus up to kb
+// pivot rows below; lu_step_perm over the whole block), so each column costs one round of loads
+// and one of stores: one warp per column, the touched rows staged in a per-warp buffer.
 __global__ void __launch_bounds__(256)
     lu_laswp_block_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
                           double* const* __restrict__ dA, const int* __restrict__ d_ld,
                           int* const* __restrict__ d_ipiv, const int* __restrict__ d_info, int batch,
                           int j0) {
-  __shared__ int srow[2 * kLuNB], ssrc[2 * kLuNB];
+  constexpr int CAP = 2 * kLuOB;
+  __shared__ int srow[CAP], ssrc[CAP];
+  __shared__ double wbuf[8][CAP];
   __shared__ int s_cnt;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   for (int i = blockIdx.x; i < batch; i += gridDim.x) {
@@ -345,25 +350,30 @@ __global__ void __launch_bounds__(256)
     const int cbeg = j0 + kLuOB;
     if (cbeg >= n || j0 >= kmax) continue;
     double* A = dA[i];
-    for (int j = j0; j < min(cbeg, kmax); j += kLuNB) {
-      const int pn = min(kLuNB, kmax - j);
-      __syncthreads();  // the previous step's columns are done with srow / ssrc
-      if (threadIdx.x == 0) s_cnt = lu_step_perm(d_ipiv[i] + j, j, pn, srow, ssrc);
-      __syncthreads();
-      const int cnt = s_cnt;
-      const int r_lo = lane < cnt ? srow[lane] : 0, r_hi = lane + 32 < cnt ? srow[lane + 32] : 0;
-      const int f_lo = lane < cnt ? ssrc[lane] : 0, f_hi = lane + 32 < cnt ? ssrc[lane + 32] : 0;
-      for (int c = cbeg + warp; c < n; c += nw) {
-        double* col = A + (size_t)c * ld;
-        const double v_lo = lane < cnt ? col[r_lo] : 0.0;
-        const double v_hi = lane + 32 < cnt ? col[r_hi] : 0.0;
-        const double a_lo = __shfl_sync(kFull, v_lo, f_lo & 31), b_lo = __shfl_sync(kFull, v_hi, f_lo & 31);
-        const double a_hi = __shfl_sync(kFull, v_lo, f_hi & 31), b_hi = __shfl_sync(kFull, v_hi, f_hi & 31);
-        if (lane < cnt) col[r_lo] = f_lo < 32 ? a_lo : b_lo;
-        if (lane + 32 < cnt) col[r_hi] = f_hi < 32 ? a_hi : b_hi;
-      }
-    }
+    const int kb = min(kLuOB, kmax - j0);
+    __syncthreads();  // the previous matrix is done with srow / ssrc
+    if (threadIdx.x == 0) s_cnt = lu_step_perm<CAP>(d_ipiv[i] + j0, j0, kb, srow, ssrc);
     __syncthreads();
+    const int cnt = s_cnt;
+    double* wb = wbuf[warp];
+    for (int c = cbeg + warp; c < n; c += nw) {
+      double* col = A + (size_t)c * ld;
+      double v[CAP / 32];
+#pragma unroll
+      for (int u = 0; u < CAP / 32; ++u) {
+        const int t = lane + 32 * u;
+        v[u] = t < cnt ? col[srow[t]] : 0.0;
+      }
+#pragma unroll
+      for (int u = 0; u < CAP / 32; ++u) wb[lane + 32 * u] = v[u];
+      __syncwarp();
+#pragma unroll
+      for (int u = 0; u < CAP / 32; ++u) {
+        const int t = lane + 32 * u;
+        if (t < cnt && ssrc[t] != t) col[srow[t]] = wb[ssrc[t]];
+      }
+      __syncwarp();
+    }
   }
 }
 
