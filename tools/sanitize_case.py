@@ -6,6 +6,8 @@ overhead, covering every kernel and protocol of one vbatched_dpotrf call (VERDIC
          roundup-32 and odd ldda (the cp.async gather instead of TMA bulk copies), failing
          pivots (-> early termination, the TMA ring drain, the look-ahead barrier exits).
   lu     vbatched_dgetrf on 40 general matrices (square and rectangular, n < 300).
+  qr     vbatched_dgeqrf on 40 general matrices (square, wide and tall).
+  host   vbatched_dpotrf_host on pinned memory in several chunks (staircase transfers).
   z      vbatched_zpotrf / vbatched_cpotrf with non-HPD matrices.
 Each case checks info against the expected values so a silent corruption also fails.
 """
@@ -68,6 +70,42 @@ def lu():
     assert np.all(lb.info() == 0)
 
 
+def qr():
+    from harness import QRBatch
+    rng = np.random.default_rng(9)
+    n = rng.integers(1, 300, 40).astype(np.int32)
+    m = n.copy()
+    m[::5] = np.maximum(1, n[::5] // 2)
+    m[1::5] = n[1::5] + 37
+    qb = QRBatch(m, n, seed=4).fill()
+    qb.geqrf()
+    torch.cuda.synchronize()
+    assert np.all(qb.info() == 0)
+
+
+def host():
+    """vbatched_dpotrf_host on pinned memory, chunked: staircase and whole-block transfers."""
+    import ctypes
+
+    import paper_conf_ipps_abdelfattahhtd16_b200 as vb
+    rng = np.random.default_rng(11)
+    n = np.concatenate([rng.integers(1, 128, 30), rng.integers(128, 400, 20)]).astype(np.int32)
+    dev = DeviceBatch(n, seed=12, nonspd_mod=7).fill(poison=True)
+    torch.cuda.synchronize()
+    src = dev.arena.cpu().numpy()
+    hp = vb.vbatched_host_alloc(src.nbytes)
+    try:
+        host = np.ctypeslib.as_array((ctypes.c_double * src.size).from_address(hp))
+        host[:] = src
+        info = np.zeros(dev.B, np.int32)
+        vb.vbatched_dpotrf_host("L", dev.n, (hp + 8 * dev.off).astype(np.int64), dev.ldda, info,
+                                dev.B, int(n.max()), workspace_bytes=3 * 4 << 20)
+        exp = np.array([vbgen.nonspd_k(12, g, int(n[g])) if g % 7 == 6 else 0 for g in range(len(n))])
+        assert np.array_equal(info, exp)
+    finally:
+        vb.vbatched_host_free(hp)
+
+
 def z():
     from harness import ZBatch
     n = np.array([1, 5, 16, 17, 40, 100, 200], np.int32)
@@ -80,5 +118,5 @@ def z():
 
 
 if __name__ == "__main__":
-    {"c1": c1, "mixed": mixed, "mixed_small": lambda: mixed(4), "mixed_gather": mixed_gather, "lu": lu, "z": z}[sys.argv[1]]()
+    {"c1": c1, "mixed": mixed, "mixed_small": lambda: mixed(4), "mixed_gather": mixed_gather, "lu": lu, "qr": qr, "host": host, "z": z}[sys.argv[1]]()
     print("case ok", sys.argv[1])
