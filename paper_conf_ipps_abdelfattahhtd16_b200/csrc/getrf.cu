@@ -123,7 +123,7 @@ __global__ void lu_block_step_kernel(const int* __restrict__ d_m, const int* __r
 // of the panel's later columns. A zero pivot (the whole column is zero) records info = j+k+1
 // (first only) and is skipped, as in DGETF2. ipiv gets the global 1-based interchanges.
 template <int RPT>
-__global__ void __launch_bounds__(kLuThreads)
+__global__ void __launch_bounds__(kLuThreads, RPT == 1 ? 3 : RPT == 2 ? 2 : 1)
     lu_panel_kernel(LuStep st, const int* __restrict__ d_ld, int* const* __restrict__ d_ipiv,
                     int* __restrict__ d_info, int batch, int j) {
   __shared__ double prow[kLuNB], krow[kLuNB];
