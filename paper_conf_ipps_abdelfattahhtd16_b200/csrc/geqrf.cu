@@ -127,7 +127,8 @@ __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
                     int batch, int j) {
   __shared__ double red[kQrThreads / 32][kQrNB];
   __shared__ double sums[kQrNB], krow[kQrNB];
-  __shared__ double s_tau[kQrNB], s_G[kQrNB][kQrNB + 1];
+  __shared__ double s_tau[kQrNB], s_G[kQrNB][kQrNB + 1], s_T[kQrNB][kQrNB + 1];
+  static_assert(kQrThreads == kQrNB * kQrNB, "one thread per entry of T");
   const int tid = threadIdx.x;
   for (int i = blockIdx.x; i < batch; i += gridDim.x) {
     const int pm = st.pm[i], pn = st.pn[i];
@@ -233,19 +234,28 @@ __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
           }
     }
     __syncthreads();
-    if (tid == 0) {  // DLARFT (forward, columnwise): T[0:i, i] = -tau_i T[0:i, 0:i] G[0:i, i]
-      double* T = st.T[i];
-      for (int e = 0; e < kQrNB * kQrNB; ++e) T[e] = 0.0;
-      for (int c = 0; c < pn; ++c) {
-        const double tc = s_tau[c];
-        for (int r = 0; r < c; ++r) {
-          double sacc = 0.0;
-          for (int q = r; q < c; ++q) sacc += T[q * kQrNB + r] * G[q][c];
-          T[c * kQrNB + r] = -tc * sacc;
+    // DLARFT (forward, columnwise): T[0:c, c] = -tau_c T[0:c, 0:c] G[0:c, c], in shared memory,
+    // thread r < 16 owning row r of T (it reads only its own row: no barrier between columns);
+    // then the whole 16 x 16 T to the workspace. (A single thread doing this through global
+    // memory was a chain of ~700 dependent L2 round trips, most of the panel kernel's time.)
+    if (tid < kQrNB) {
+      const int r = tid;
+      for (int c = 0; c < kQrNB; ++c) {
+        double v = 0.0;
+        if (c < pn) {
+          if (r < c) {
+            double sacc = 0.0;
+            for (int q = r; q < c; ++q) sacc += s_T[q][r] * G[q][c];
+            v = -s_tau[c] * sacc;
+          } else if (r == c) {
+            v = s_tau[c];
+          }
         }
-        T[c * kQrNB + c] = tc;
+        s_T[c][r] = v;
       }
     }
+    __syncthreads();
+    st.T[i][tid] = s_T[tid / kQrNB][tid % kQrNB];  // kQrThreads == 16 x 16
     __syncthreads();
   }
 }
