@@ -102,21 +102,45 @@ __global__ void qr_step_kernel(const int* __restrict__ d_m, const int* __restric
   }
 }
 
-// Block-wide sums of 16 per-thread partials (all threads get them in `out`).
+// Block-wide sums of 16 per-thread partials (all threads get them in `out`). Within a warp by
+// recursive halving: at each of the exchange levels 16, 8, 4, 2 a lane keeps one half of its
+// values and adds the partner's copy of that half (8 + 4 + 2 + 1 shuffles instead of 16 x 5),
+// after which lane l holds value 8 b4 + 4 b3 + 2 b2 + b1 (b_i = bit i of l) summed over the warp
+// (lanes l and l ^ 1 alike). Across the 8 warps: 128 threads, one per (value, warp), 3 shuffles.
 VB_DEVINL void block_sum16(double (&p)[kQrNB], double (*red)[kQrNB], double* out, int tid) {
+  static_assert(kQrNB == 16 && kQrThreads == 256, "shapes");
   const int lane = tid & 31, warp = tid >> 5;
+  double v8[8], v4[4], v2[2];
+  bool hi = lane & 16;
 #pragma unroll
-  for (int c = 0; c < kQrNB; ++c)
+  for (int k = 0; k < 8; ++k) {
+    const double send = hi ? p[k] : p[k + 8], keep = hi ? p[k + 8] : p[k];
+    v8[k] = keep + __shfl_xor_sync(kFull, send, 16);
+  }
+  hi = lane & 8;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) p[c] += __shfl_xor_sync(kFull, p[c], o);
-  if (lane == 0)
+  for (int k = 0; k < 4; ++k) {
+    const double send = hi ? v8[k] : v8[k + 4], keep = hi ? v8[k + 4] : v8[k];
+    v4[k] = keep + __shfl_xor_sync(kFull, send, 8);
+  }
+  hi = lane & 4;
 #pragma unroll
-    for (int c = 0; c < kQrNB; ++c) red[warp][c] = p[c];
+  for (int k = 0; k < 2; ++k) {
+    const double send = hi ? v4[k] : v4[k + 2], keep = hi ? v4[k + 2] : v4[k];
+    v2[k] = keep + __shfl_xor_sync(kFull, send, 4);
+  }
+  hi = lane & 2;
+  double v1 = (hi ? v2[1] : v2[0]) + __shfl_xor_sync(kFull, hi ? v2[0] : v2[1], 2);
+  v1 += __shfl_xor_sync(kFull, v1, 1);
+  const int idx = ((lane >> 4) & 1) * 8 + ((lane >> 3) & 1) * 4 + ((lane >> 2) & 1) * 2 + ((lane >> 1) & 1);
+  if ((lane & 1) == 0) red[warp][idx] = v1;
   __syncthreads();
-  if (tid < kQrNB) {
-    double s = 0.0;
-    for (int w = 0; w < kQrThreads / 32; ++w) s += red[w][tid];
-    out[tid] = s;
+  if (tid < 128) {
+    double x = red[tid & 7][tid >> 3];
+    x += __shfl_xor_sync(kFull, x, 1);
+    x += __shfl_xor_sync(kFull, x, 2);
+    x += __shfl_xor_sync(kFull, x, 4);
+    if ((tid & 7) == 0) out[tid >> 3] = x;
   }
   __syncthreads();
 }
