@@ -35,7 +35,10 @@ static cudaError_t lib_pool(cudaMemPool_t* out) {
     props.location.id = dev;
     cudaMemPool_t p;
     if ((e = cudaMemPoolCreate(&p, &props)) != cudaSuccess) return e;
-    uint64_t thr = 256ull << 20;
+    // Workspace stays mapped between calls up to 8 GiB: with a small threshold the pool trims
+    // at every synchronisation and the next call re-maps its workspace (GEQRF's is ~0.8 GB for
+    // 3000 x 512 and took 47 or 62 ms per call depending on whether it had been trimmed).
+    uint64_t thr = 8ull << 30;
     cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
     g_pool[dev] = p;
   }
