@@ -2,15 +2,19 @@
 // names as future work (§V; §III-E), built from the same
 // vbatched kernels in the paper's separated style.
 //
-// Per panel of NB = 16 columns (LAPACK DGEQRF's blocked algorithm):
+// LAPACK DGEQRF's blocked algorithm in two levels, so that the trailing matrix is streamed three
+// times per 64 columns instead of per 16 (its updates are HBM-bound). Per 16-column step j of a
+// 64-column block [j0, j0 + 64):
 //   step kernel   per-matrix sub-problem sizes and pointers, on the GPU;
 //   panel kernel  DGEQR2 on the panel with the rows in registers (one CTA per matrix): per
 //                 column one block reduction gives ||x||^2 and the 15 dot products the
-//                 reflector needs; then V (unit lower, explicit) and the triangular factor T of
-//                 the block reflector H_1..H_nb = I - V T V^T (DLARFT, forward, columnwise) go to
-//                 the workspace;
-//   trailing      A2 <- (I - V T V^T)^T A2 = A2 - V (T^T (V^T A2)) as three calls of the
-//                 library's vbatched DGEMM (DMMA): W1 = V^T A2, W2 = T^T W1, A2 -= V W2.
+//                 reflector needs; then V (unit lower, explicit) goes to the block's V in the
+//                 workspace and the triangular factor T of the panel's block reflector
+//                 H_1..H_nb = I - V T V^T (DLARFT, forward, columnwise) next to it;
+//   block update  A2 <- (I - V T V^T)^T A2 = A2 - V (T^T (V^T A2)) on the block's columns right
+//                 of the panel, three calls of the library's vbatched DGEMM (DMMA).
+// After the block: G = Vb^T Vb (vbatched DGEMM), the block's 64 x 64 T from G and tau (DLARFT,
+// qr_larft_kernel), and the same three GEMMs with k = 64 on the trailing columns.
 #include <algorithm>
 
 #include "../../include/vbatched.h"
@@ -21,20 +25,29 @@ namespace vb {
 namespace {
 
 constexpr int kQrNB = 16;
+constexpr int kQrOB = 64;  // outer block width
 constexpr int kQrThreads = 256;
 constexpr int kQrMaxRPT = 4;  // panel rows in registers: m - j <= 1024
 
 struct QrStep {
-  int *pm, *pn, *rn, *vld, *sixteen;
+  int *pm, *pn, *rn, *vld, *sixteen, *sixtyfour;
   double **P, **A2, **V, **W1, **W2, **T;
+  // after a block: kb reflectors, bm = m - j0 rows, bn trailing columns
+  int *kb, *bm, *bn;
+  double **Vb, **G, **Tb, **A2b;
 };
+// per-matrix workspace (doubles): V 64 m | W1 64 n | W2 64 n | T 16 x 16 | Tb 64 x 64 | G 64 x 64
+VB_DEVINL size_t qr_ws_doubles(int m, int n) {
+  return (size_t)kQrOB * m + 2 * (size_t)kQrOB * n + kQrNB * kQrNB + 2 * kQrOB * kQrOB;
+}
 
 // info: -1 m < 0, -2 n < 0, -4 ldda < max(1, m), -9 beyond max_m / max_n; workspace offsets
 // (16 m + 32 n + 256 doubles per matrix) by an exclusive prefix sum in one CTA.
 __global__ void __launch_bounds__(1024, 1)
     qr_prep_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
                    const int* __restrict__ d_ld, int* __restrict__ d_info, int batch, int max_m,
-                   int max_n, size_t* __restrict__ woff, int* __restrict__ sixteen) {
+                   int max_n, size_t* __restrict__ woff, int* __restrict__ sixteen,
+                   int* __restrict__ sixtyfour) {
   __shared__ size_t wsum[32];
   __shared__ size_t carry;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -52,7 +65,8 @@ __global__ void __launch_bounds__(1024, 1)
       else if (m > max_m || n > max_n) code = -9;
       d_info[i] = code;
       sixteen[i] = kQrNB;
-      if (code == 0) sz = 16 * (size_t)m + 32 * (size_t)n + 256;
+      sixtyfour[i] = kQrOB;
+      if (code == 0) sz = qr_ws_doubles(m, n);
     }
     size_t incl = sz;
     for (int o = 1; o < 32; o <<= 1) {
@@ -81,24 +95,84 @@ __global__ void __launch_bounds__(1024, 1)
 __global__ void qr_step_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
                                double* const* __restrict__ dA, const int* __restrict__ d_ld,
                                const int* __restrict__ d_info, const size_t* __restrict__ woff,
-                               double* __restrict__ wbase, int batch, int j, QrStep st) {
+                               double* __restrict__ wbase, int batch, int j, int j0, QrStep st) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
     const int m = d_m[i], n = d_n[i], ld = d_ld[i];
     const int kmax = m < n ? m : n;
     const bool act = d_info[i] >= 0 && j < kmax;
     const int nb = act ? min(kQrNB, kmax - j) : 0;
+    const int cend = min(j0 + kQrOB, n);  // the block's columns only
     st.pm[i] = act ? m - j : 0;
     st.pn[i] = nb;
-    st.rn[i] = act ? n - j - nb : 0;
-    st.vld[i] = act ? m - j : 1;
+    st.rn[i] = act ? max(0, cend - j - nb) : 0;
+    st.vld[i] = act ? m - j0 : 1;
     double* A = dA[i];
     double* w = wbase + woff[i];
+    const size_t mm = (size_t)max(m, 0), nn = (size_t)max(n, 0);
     st.P[i] = act ? A + (size_t)j * ld + j : A;
     st.A2[i] = act ? A + (size_t)(j + nb) * ld + j : A;
-    st.V[i] = w;                                  // 16 m doubles (ld m - j this step)
-    st.W1[i] = w + 16 * (size_t)max(m, 0);        // 16 n
-    st.W2[i] = st.W1[i] + 16 * (size_t)max(n, 0); // 16 n
-    st.T[i] = st.W2[i] + 16 * (size_t)max(n, 0);  // 16 x 16
+    // the block's V (ld m - j0): this panel's columns start at (j - j0, j - j0)
+    st.V[i] = act ? w + (size_t)(j - j0) * (m - j0) + (j - j0) : w;
+    st.W1[i] = w + kQrOB * mm;
+    st.W2[i] = st.W1[i] + kQrOB * nn;
+    st.T[i] = st.W2[i] + kQrOB * nn;  // 16 x 16
+  }
+}
+
+// After the block [j0, j0 + 64): pointers and sizes of G = Vb^T Vb, the block T and the trailing
+// update (rows j0.., columns j0 + 64..).
+__global__ void qr_block_step_kernel(const int* __restrict__ d_m, const int* __restrict__ d_n,
+                                     double* const* __restrict__ dA, const int* __restrict__ d_ld,
+                                     const int* __restrict__ d_info, const size_t* __restrict__ woff,
+                                     double* __restrict__ wbase, int batch, int j0, QrStep st) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < batch; i += gridDim.x * blockDim.x) {
+    const int m = d_m[i], n = d_n[i], ld = d_ld[i];
+    const int kmax = m < n ? m : n;
+    const int e = j0 + kQrOB;
+    const bool act = d_info[i] >= 0 && j0 < kmax && e < n;
+    double* A = dA[i];
+    double* w = wbase + woff[i];
+    const size_t mm = (size_t)max(m, 0), nn = (size_t)max(n, 0);
+    st.kb[i] = act ? min(kQrOB, kmax - j0) : 0;
+    st.bm[i] = act ? m - j0 : 0;
+    st.bn[i] = act ? n - e : 0;
+    st.vld[i] = act ? m - j0 : 1;
+    st.Vb[i] = w;
+    st.W1[i] = w + kQrOB * mm;
+    st.W2[i] = st.W1[i] + kQrOB * nn;
+    st.Tb[i] = st.W2[i] + kQrOB * nn + kQrNB * kQrNB;
+    st.G[i] = st.Tb[i] + kQrOB * kQrOB;
+    st.A2b[i] = act ? A + (size_t)e * ld + j0 : A;
+  }
+}
+
+// The block reflector's T (kb x kb, ld 64) from G = Vb^T Vb and tau (LAPACK DLARFT, forward,
+// columnwise): T(c, c) = tau_c, T(0:c, c) = -tau_c T(0:c, 0:c) G(0:c, c). One CTA per matrix,
+// thread r owns row r; one barrier per column.
+__global__ void __launch_bounds__(64)
+    qr_larft_kernel(QrStep st, double* const* __restrict__ d_tau, int batch, int j0) {
+  __shared__ double T[kQrOB][kQrOB + 1];  // T[col][row]
+  const int r = threadIdx.x;
+  for (int i = blockIdx.x; i < batch; i += gridDim.x) {
+    const int kb = st.kb[i];
+    if (kb <= 0) continue;
+    const double* G = st.G[i];
+    const double* tau = d_tau[i] + j0;
+    for (int c = 0; c < kb; ++c) {
+      double v = 0.0;
+      if (r < c) {
+        double sacc = 0.0;
+        for (int q = r; q < c; ++q) sacc = fma(T[q][r], G[(size_t)c * kQrOB + q], sacc);
+        v = -tau[c] * sacc;
+      } else if (r == c) {
+        v = tau[c];
+      }
+      T[c][r] = v;
+      __syncthreads();
+    }
+    double* Tg = st.Tb[i];
+    for (int c = 0; c < kb; ++c) Tg[(size_t)c * kQrOB + r] = r < kb ? T[c][r] : 0.0;
+    __syncthreads();
   }
 }
 
@@ -148,7 +222,7 @@ VB_DEVINL void block_sum16(double (&p)[kQrNB], double (*red)[kQrNB], double* out
 template <int RPT>
 __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
     qr_panel_kernel(QrStep st, const int* __restrict__ d_ld, double* const* __restrict__ d_tau,
-                    int batch, int j) {
+                    int batch, int j, int j0) {
   __shared__ double red[kQrThreads / 32][kQrNB];
   __shared__ double sums[kQrNB], krow[kQrNB];
   __shared__ double s_tau[kQrNB], s_G[kQrNB][kQrNB + 1], s_T[kQrNB][kQrNB + 1];
@@ -224,6 +298,12 @@ __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
     // panel back to global (R on/above the diagonal, v below); V (unit lower, explicit) to the
     // workspace; partial Gram sums V^T V for DLARFT
     double* V = st.V[i];
+    const int vld = st.vld[i];
+    {  // the block's rows above this panel are zero in its V columns
+      const int top = j - j0;
+      for (int e = tid; e < top * pn; e += kQrThreads)
+        V[(size_t)(e / top) * vld - top + e % top] = 0.0;
+    }
     double g[kQrNB];
 #pragma unroll
     for (int c = 0; c < kQrNB; ++c) g[c] = 0.0;
@@ -254,7 +334,7 @@ __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
         for (int c = 0; c < kQrNB; ++c)
           if (c < pn) {
             P[(size_t)c * ld + r] = a[s][c];
-            V[(size_t)c * pm + r] = (r == c) ? 1.0 : (r < c ? 0.0 : a[s][c]);
+            V[(size_t)c * vld + r] = (r == c) ? 1.0 : (r < c ? 0.0 : a[s][c]);
           }
     }
     __syncthreads();
@@ -286,8 +366,8 @@ __global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
 
 template <int RPT>
 cudaError_t launch_qr_panel(int grid, QrStep st, const int* d_ld, double* const* d_tau, int batch,
-                            int j, cudaStream_t stream) {
-  qr_panel_kernel<RPT><<<grid, kQrThreads, 0, stream>>>(st, d_ld, d_tau, batch, j);
+                            int j, int j0, cudaStream_t stream) {
+  qr_panel_kernel<RPT><<<grid, kQrThreads, 0, stream>>>(st, d_ld, d_tau, batch, j, j0);
   return cudaGetLastError();
 }
 
@@ -300,9 +380,10 @@ int geqrf_impl(const int* d_m, const int* d_n, double* const* dA, const int* d_l
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   // host-side upper bound of the per-matrix workspace (the device prefix sum fills it exactly)
-  const size_t wdoubles = (size_t)batch * (16 * (size_t)max_m + 32 * (size_t)max_n + 256);
+  const size_t wdoubles = (size_t)batch * ((size_t)kQrOB * max_m + 2 * (size_t)kQrOB * max_n +
+                                           kQrNB * kQrNB + 2 * kQrOB * kQrOB);
   const size_t ib = sizeof(int) * (size_t)batch, pb = sizeof(double*) * (size_t)batch;
-  const size_t meta = 5 * ib + 6 * pb + sizeof(size_t) * (size_t)batch;
+  const size_t meta = 9 * ib + 10 * pb + sizeof(size_t) * (size_t)batch;
   void* ws = nullptr;
   cudaError_t e = ws_alloc(&ws, ((meta + 255) & ~(size_t)255) + 8 * wdoubles, stream);
   if (e != cudaSuccess) return (int)e;
@@ -314,40 +395,72 @@ int geqrf_impl(const int* d_m, const int* d_n, double* const* dA, const int* d_l
   st.W1 = st.V + batch;
   st.W2 = st.W1 + batch;
   st.T = st.W2 + batch;
-  size_t* woff = reinterpret_cast<size_t*>(st.T + batch);
+  st.Vb = st.T + batch;
+  st.G = st.Vb + batch;
+  st.Tb = st.G + batch;
+  st.A2b = st.Tb + batch;
+  size_t* woff = reinterpret_cast<size_t*>(st.A2b + batch);
   st.pm = reinterpret_cast<int*>(woff + batch);
   st.pn = st.pm + batch;
   st.rn = st.pn + batch;
   st.vld = st.rn + batch;
   st.sixteen = st.vld + batch;
+  st.sixtyfour = st.sixteen + batch;
+  st.kb = st.sixtyfour + batch;
+  st.bm = st.kb + batch;
+  st.bn = st.bm + batch;
   double* wbase = reinterpret_cast<double*>(w + ((meta + 255) & ~(size_t)255));
   qr_prep_kernel<<<1, 1024, 0, stream>>>(d_m, d_n, d_ld, d_info, batch, max_m, max_n, woff,
-                                         st.sixteen);
+                                         st.sixteen, st.sixtyfour);
   e = cudaGetLastError();
   const int eg = std::max(1, std::min((batch + 255) / 256, 4 * sms));
   const int pg = std::max(1, std::min(batch, 8 * sms));
   const int kmax = std::min(max_m, max_n);
-  for (int j = 0; j < kmax && e == cudaSuccess; j += kQrNB) {
-    qr_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, woff, wbase, batch, j, st);
-    if ((e = cudaGetLastError()) != cudaSuccess) break;
-    const int rows = max_m - j;
-    if (rows <= kQrThreads) e = launch_qr_panel<1>(pg, st, d_ld, d_tau, batch, j, stream);
-    else if (rows <= 2 * kQrThreads) e = launch_qr_panel<2>(pg, st, d_ld, d_tau, batch, j, stream);
-    else e = launch_qr_panel<4>(pg, st, d_ld, d_tau, batch, j, stream);
-    if (e != cudaSuccess) break;
-    if (j + kQrNB < max_n) {  // trailing update with the block reflector
-      int rc = gemm_launch('T', 'N', st.pn, st.rn, st.pm, 1.0, st.V, st.vld, st.A2, d_ld, 0.0,
-                           st.W1, st.sixteen, batch, kQrNB, max_n, max_m, stream);
-      if (rc == 0)
-        rc = gemm_launch('T', 'N', st.pn, st.rn, st.pn, 1.0, st.T, st.sixteen, st.W1, st.sixteen,
-                         0.0, st.W2, st.sixteen, batch, kQrNB, max_n, kQrNB, stream);
-      if (rc == 0)
-        rc = gemm_launch('N', 'N', st.pm, st.rn, st.pn, -1.0, st.V, st.vld, st.W2, st.sixteen, 1.0,
-                         st.A2, d_ld, batch, max_m, max_n, kQrNB, stream);
-      if (rc != 0) {
-        e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
-        break;
+  for (int j0 = 0; j0 < kmax && e == cudaSuccess; j0 += kQrOB) {
+    for (int j = j0; j < std::min(j0 + kQrOB, kmax) && e == cudaSuccess; j += kQrNB) {
+      qr_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, woff, wbase, batch, j, j0, st);
+      if ((e = cudaGetLastError()) != cudaSuccess) break;
+      const int rows = max_m - j;
+      if (rows <= kQrThreads) e = launch_qr_panel<1>(pg, st, d_ld, d_tau, batch, j, j0, stream);
+      else if (rows <= 2 * kQrThreads) e = launch_qr_panel<2>(pg, st, d_ld, d_tau, batch, j, j0, stream);
+      else e = launch_qr_panel<4>(pg, st, d_ld, d_tau, batch, j, j0, stream);
+      if (e != cudaSuccess) break;
+      // the block's columns right of the panel (a last panel narrower than 16 columns still has
+      // the block's remaining columns on its right)
+      if (j + 1 < std::min(j0 + kQrOB, max_n)) {
+        int rc = gemm_launch('T', 'N', st.pn, st.rn, st.pm, 1.0, st.V, st.vld, st.A2, d_ld, 0.0,
+                             st.W1, st.sixteen, batch, kQrNB, kQrOB, max_m, stream);
+        if (rc == 0)
+          rc = gemm_launch('T', 'N', st.pn, st.rn, st.pn, 1.0, st.T, st.sixteen, st.W1, st.sixteen,
+                           0.0, st.W2, st.sixteen, batch, kQrNB, kQrOB, kQrNB, stream);
+        if (rc == 0)
+          rc = gemm_launch('N', 'N', st.pm, st.rn, st.pn, -1.0, st.V, st.vld, st.W2, st.sixteen, 1.0,
+                           st.A2, d_ld, batch, max_m, kQrOB, kQrNB, stream);
+        if (rc != 0) {
+          e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
+          break;
+        }
       }
+    }
+    if (e == cudaSuccess && j0 + kQrOB < max_n) {  // the block reflector on the trailing columns
+      qr_block_step_kernel<<<eg, 256, 0, stream>>>(d_m, d_n, dA, d_ld, d_info, woff, wbase, batch,
+                                                   j0, st);
+      if ((e = cudaGetLastError()) != cudaSuccess) break;
+      int rc = gemm_launch('T', 'N', st.kb, st.kb, st.bm, 1.0, st.Vb, st.vld, st.Vb, st.vld, 0.0,
+                           st.G, st.sixtyfour, batch, kQrOB, kQrOB, max_m, stream);
+      if (rc == 0) {
+        qr_larft_kernel<<<pg, 64, 0, stream>>>(st, d_tau, batch, j0);
+        if ((e = cudaGetLastError()) != cudaSuccess) break;
+        rc = gemm_launch('T', 'N', st.kb, st.bn, st.bm, 1.0, st.Vb, st.vld, st.A2b, d_ld, 0.0,
+                         st.W1, st.sixtyfour, batch, kQrOB, max_n, max_m, stream);
+      }
+      if (rc == 0)
+        rc = gemm_launch('T', 'N', st.kb, st.bn, st.kb, 1.0, st.Tb, st.sixtyfour, st.W1,
+                         st.sixtyfour, 0.0, st.W2, st.sixtyfour, batch, kQrOB, max_n, kQrOB, stream);
+      if (rc == 0)
+        rc = gemm_launch('N', 'N', st.bm, st.bn, st.kb, -1.0, st.Vb, st.vld, st.W2, st.sixtyfour,
+                         1.0, st.A2b, d_ld, batch, max_m, max_n, kQrOB, stream);
+      if (rc != 0) e = rc > 0 ? (cudaError_t)rc : cudaErrorInvalidValue;
     }
   }
   cudaError_t e2 = ws_free(ws, stream);
