@@ -220,7 +220,7 @@ VB_DEVINL void block_sum16(double (&p)[kQrNB], double (*red)[kQrNB], double* out
 }
 
 template <int RPT>
-__global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : 1)
+__global__ void __launch_bounds__(kQrThreads, RPT == 1 ? 3 : RPT == 2 ? 2 : 1)
     qr_panel_kernel(QrStep st, const int* __restrict__ d_ld, double* const* __restrict__ d_tau,
                     int batch, int j, int j0) {
   __shared__ double red[kQrThreads / 32][kQrNB];
