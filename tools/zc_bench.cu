@@ -56,6 +56,51 @@ int main() {
   };
   rep("memcpy H2D (copy engine)", [&] { cudaMemcpyAsync(d, h, bytes, cudaMemcpyHostToDevice); });
   rep("memcpy D2H (copy engine)", [&] { cudaMemcpyAsync(h, d, bytes, cudaMemcpyDeviceToHost); });
+  {  // both directions at once on two streams (H2D of one buffer, D2H of another)
+    double *h2, *d2;
+    cudaHostAlloc(&h2, bytes, cudaHostAllocDefault);
+    cudaMalloc(&d2, bytes);
+    cudaStream_t s1, s2;
+    cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking);
+    cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking);
+    for (int it = 0; it < 2; ++it) {
+      cudaDeviceSynchronize();
+      cudaEventRecord(e0);
+      cudaEventRecord(e0, 0);
+      cudaStreamWaitEvent(s1, e0, 0);
+      cudaStreamWaitEvent(s2, e0, 0);
+      cudaMemcpyAsync(d, h, bytes, cudaMemcpyHostToDevice, s1);
+      cudaMemcpyAsync(h2, d2, bytes, cudaMemcpyDeviceToHost, s2);
+      cudaEvent_t a, b;
+      cudaEventCreate(&a);
+      cudaEventCreate(&b);
+      cudaEventRecord(a, s1);
+      cudaEventRecord(b, s2);
+      cudaStreamWaitEvent(0, a, 0);
+      cudaStreamWaitEvent(0, b, 0);
+      cudaEventRecord(e1, 0);
+      cudaEventSynchronize(e1);
+      float ms;
+      cudaEventElapsedTime(&ms, e0, e1);
+      if (it) printf("{\"op\":\"memcpy H2D + D2H concurrently (copy engines)\",\"GBps_each\":%.1f,\"GBps_total\":%.1f}\n",
+                     bytes / ms / 1e6, 2 * bytes / ms / 1e6);
+    }
+    fflush(stdout);
+  }
+  for (size_t w : {1024, 2048, 4096, 6144}) {  // 2-D copies: rows of w bytes at an 8 KiB pitch
+    char name[96];
+    snprintf(name, sizeof name, "memcpy2D H2D width %zu B pitch 8192 B (GB/s of payload)", w);
+    const size_t rows = bytes / 8192;
+    cudaDeviceSynchronize();
+    cudaEventRecord(e0);
+    cudaMemcpy2DAsync(d, 8192, h, 8192, w, rows, cudaMemcpyHostToDevice);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    printf("{\"op\":\"%s\",\"GBps\":%.1f}\n", name, rows * w / ms / 1e6);
+    fflush(stdout);
+  }
   rep("kernel read 8B ldcv x4, 2x128/SM", [&] { zc_read<1, 4, 0><<<2 * sms, 128>>>(h, d, n); });
   rep("kernel read 16B ldcv x4, 2x128/SM", [&] { zc_read<2, 4, 0><<<2 * sms, 128>>>(h, d, n); });
   rep("kernel read 16B ldcg x4, 2x128/SM", [&] { zc_read<2, 4, 1><<<2 * sms, 128>>>(h, d, n); });
