@@ -45,6 +45,10 @@
 namespace vb {
 
 // Every other row block of a panel walks the k chunks backwards (produce_matrix3); 0 disables.
+// Small-kernel CTAs per SM (launch bounds and grid).
+#ifndef VB_SMALL_CPS
+#define VB_SMALL_CPS 4
+#endif
 #ifndef VB_KREV
 #define VB_KREV 1
 #endif
@@ -1225,7 +1229,7 @@ VB_DEVINL void la_matrix_v2(SmallSmem& s, int role, int lane, E* __restrict__ A,
 // with the off-diagonal DMMA streams (tools/contention_bench.cu: a DMMA stream starves the
 // FP64 chain on its sub-partition). Each pair fetches its own matrices.
 template <bool UP, typename E = double>
-__global__ void __launch_bounds__(128, 4)
+__global__ void __launch_bounds__(128, VB_SMALL_CPS)
     potrf_small_kernel(const int* __restrict__ d_n, E* const* __restrict__ dA,
                            const int* __restrict__ d_ldda, int* __restrict__ d_info,
                            const Ctrl* __restrict__ ctrl_c, const int* __restrict__ order,
@@ -1447,7 +1451,7 @@ static cudaError_t launch_paths(const int* d_n, E* const* dA, const int* d_ldda,
   const int sms = g_num_sms.load();
   if (max_n_hint > kWarpMaxN) {
     cfg.blockDim = dim3(128);
-    cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, sms * 4)));
+    cfg.gridDim = dim3(std::max(1, std::min((batch + 1) / 2, sms * VB_SMALL_CPS)));
     cfg.dynamicSmemBytes = 0;
     e = cudaLaunchKernelEx(&cfg, up ? potrf_small_kernel<true, E> : potrf_small_kernel<false, E>,
                            d_n, dA, d_ldda, d_info, ctrl, order, 1, wait);
@@ -1478,7 +1482,7 @@ void potrf_occupancy(int* out4) {
   out4[0] = g_occ64.load();
   out4[1] = Cfg64d::WARPS;
   out4[2] = 0;  // (no separate NB=32 range)
-  out4[3] = 4;  // small kernel: 4 CTAs (8 matrices) per SM
+  out4[3] = VB_SMALL_CPS;  // small kernel: CTAs (2 matrices each) per SM
 }
 
 int potrf_num_launches(int max_n_hint) {
