@@ -49,6 +49,10 @@ namespace vb {
 #ifndef VB_SMALL_CPS
 #define VB_SMALL_CPS 4
 #endif
+// L2 prefetch distance of the blocked kernel's A chunks (0: none).
+#ifndef VB_PF
+#define VB_PF 0
+#endif
 #ifndef VB_KREV
 #define VB_KREV 1
 #endif
@@ -599,7 +603,17 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const typename C::E* A, int n, int l
       const int rn = (min(MB, n - j0) + G - 1) / G * G;
       bulk_prefetch_l2(A + (size_t)(j0 + lane) * ld + j0, rn * (int)sizeof(E));
     }
-    for (int kc = 0; kc < nk_free; ++kc) issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
+    // L2 prefetch of the A chunk VB_PF chunks ahead of the one being issued (the ring holds one)
+    auto pf = [&](int r0, int kcp, int lim) {
+      if (VB_PF > 0 && bulk && kcp >= 0 && kcp < lim && lane < KC) {
+        const int ra = (min(MB, n - r0) + G - 1) / G * G;
+        bulk_prefetch_l2(A + (size_t)(kcp * KC + lane) * ld + r0, ra * (int)sizeof(E));
+      }
+    };
+    for (int kc = 0; kc < nk_free; ++kc) {
+      pf(j0, kc + VB_PF, nk_free);
+      issue_chunk2<C, UP>(s, gchunk++, kc, A, n, ld, j0, j0, lane, bulk);
+    }
     if (lane == 0) mbar_wait(&s.panel_done, (gpanel + p - 1) & 1);  // panel p-1 is stored
     __syncwarp();
     if (s.info) {  // the consumers failed in panel p-1 and stop there (they also drain the
@@ -614,8 +628,10 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const typename C::E* A, int n, int l
       // Every other row block walks the k chunks backwards, so the panel rows' chunks it reads
       // first are the ones the previous block read last (still in L2)
       const bool rev = VB_KREV && (((r0 - j0) / MB) & 1);
-      for (int i = (r0 == j0 ? nk_free : 0); i < nk; ++i)
+      for (int i = (r0 == j0 ? nk_free : 0); i < nk; ++i) {
+        pf(r0, rev ? nk - 1 - (i + VB_PF) : i + VB_PF, nk);
         issue_chunk2<C, UP>(s, gchunk++, rev ? nk - 1 - i : i, A, n, ld, r0, j0, lane, bulk);
+      }
     }
   }
   gpanel += done;
