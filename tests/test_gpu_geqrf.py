@@ -69,3 +69,19 @@ def test_geqrf_mixed_batch():
     qb = QRBatch(m, n, seed=73).fill()
     qb.geqrf()
     _check(qb, idxs=range(0, 300, 4))
+
+
+# the two-level blocking's edges (16-column steps inside 64-column blocks): block boundaries in m,
+# n and min(m, n); a last block narrower than 64 with trailing columns (wide), a full block with no
+# rows below it, tall matrices ending on a block
+BLOCK_EDGES = [(63, 63), (64, 200), (200, 64), (65, 130), (130, 65), (70, 130), (130, 70),
+               (127, 129), (129, 127), (191, 192), (192, 193), (193, 191), (250, 70), (70, 250)]
+
+
+@pytest.mark.parametrize("pad", [0, 3])
+def test_geqrf_block_edges(pad):
+    m = np.array([s[0] for s in BLOCK_EDGES], np.int32)
+    n = np.array([s[1] for s in BLOCK_EDGES], np.int32)
+    qb = QRBatch(m, n, seed=44, ldda=np.maximum(1, m) + pad).fill()
+    qb.geqrf()
+    _check(qb)

@@ -125,3 +125,20 @@ def test_getrf_stream_and_repeat_bit_identical():
     assert torch.equal(a.ipiv, b.ipiv)
     for i in range(a.B):
         assert np.array_equal(a.block(i).view(np.uint64), b.block(i).view(np.uint64)), i
+
+
+# the two-level blocking's edges (SURVEY §8(f) NEXT-4 built with 16-column steps inside 64-column
+# blocks): block boundaries in m, n and min(m, n); a last block narrower than 64 with trailing
+# columns (wide), a full block with no rows below it (kmax = 64), tall matrices ending on a block
+BLOCK_EDGES = [(63, 63), (64, 200), (200, 64), (65, 130), (130, 65), (70, 130), (130, 70),
+               (127, 129), (129, 127), (191, 192), (192, 193), (193, 191), (250, 70), (70, 250)]
+
+
+@pytest.mark.parametrize("pad", [0, 3])
+def test_getrf_block_edges(pad):
+    m = np.array([s[0] for s in BLOCK_EDGES], np.int32)
+    n = np.array([s[1] for s in BLOCK_EDGES], np.int32)
+    lb = LUBatch(m, n, seed=43, ldda=np.maximum(1, m) + pad).fill()
+    lb.getrf()
+    info = _check_all(lb)
+    assert np.all(info == 0)
