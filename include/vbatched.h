@@ -244,7 +244,8 @@ int vbatched_dgetrf(const int* d_m, const int* d_n, double* const* dA_array, con
  *  max_m, max_n bounds (host); max_m <= 1024 (panel rows in registers), larger returns -8.
  * Reflectors: LAPACK DLARFG conventions (beta = -sign(alpha) sqrt(alpha^2 + ||x||^2), tau =
  * (beta - alpha)/beta, v = x/(alpha - beta); ||x|| = 0 gives tau = 0). Internal workspace:
- * batchCount x (16 max_m + 32 max_n + 256) doubles from the library's pool for the call.
+ * (64 max_m + 128 max_n + 8448) doubles per matrix from the library's pool, the batch processed
+ * in slices of at most ~4 GiB of workspace.
  * Returns 0 / -p (batchCount -7, max_m -8, max_n -9) / cudaError_t.
  */
 int vbatched_dgeqrf(const int* d_m, const int* d_n, double* const* dA_array, const int* d_ldda,

@@ -478,6 +478,17 @@ extern "C" int vbatched_dgeqrf(const int* d_m, const int* d_n, double* const* dA
   if (max_m < 0) return -8;
   if (max_n < 0) return -9;
   if (batchCount == 0) return 0;
-  return geqrf_impl(d_m, d_n, dA_array, d_ldda, dtau_array, d_info, batchCount, max_m, max_n,
-                    (cudaStream_t)stream);
+  // The per-matrix workspace (64 m + 128 n + 8448 doubles at the bounds: 1.5 MB for 1024 x 1024)
+  // is bounded to ~4 GiB per call by slicing the batch; matrices are independent, so a slice is
+  // the same call on a sub-range of the arrays.
+  const size_t per = ((size_t)kQrOB * max_m + 2 * (size_t)kQrOB * max_n + kQrNB * kQrNB +
+                      2 * kQrOB * kQrOB) * sizeof(double) + 256;
+  const int slice = (int)std::max<size_t>(1, std::min<size_t>(batchCount, (4ull << 30) / per));
+  for (int b0 = 0; b0 < batchCount; b0 += slice) {
+    const int cnt = std::min(slice, batchCount - b0);
+    const int rc = geqrf_impl(d_m + b0, d_n + b0, dA_array + b0, d_ldda + b0, dtau_array + b0,
+                              d_info + b0, cnt, max_m, max_n, (cudaStream_t)stream);
+    if (rc != 0) return rc;
+  }
+  return 0;
 }

@@ -85,3 +85,14 @@ def test_geqrf_block_edges(pad):
     qb = QRBatch(m, n, seed=44, ldda=np.maximum(1, m) + pad).fill()
     qb.geqrf()
     _check(qb)
+
+
+def test_geqrf_sliced_batch():
+    """More matrices than one ~4 GiB workspace slice at the declared bounds (1024 x 1024): the
+    batch runs as several slices, every matrix still factored (sampled against the oracle)."""
+    rng = np.random.default_rng(45)
+    n = rng.integers(1, 40, 3000).astype(np.int32)
+    m = (n + rng.integers(0, 20, 3000)).astype(np.int32)
+    qb = QRBatch(m, n, seed=46).fill()
+    qb.geqrf(max_m=1024, max_n=1024)
+    _check(qb, idxs=list(range(0, 3000, 97)) + [2599, 2600, 2601, 2999])
