@@ -18,7 +18,8 @@
  *    synchronisation and no device->host copy happens unless the routine says so. Internal
  *    workspace (O(batchCount) ints) is stream-ordered (cudaMallocFromPoolAsync/cudaFreeAsync
  *    on a memory pool the library creates per device; the caller's default pool and its
- *    attributes are not touched).
+ *    attributes are not touched). The library's pool keeps up to 8 GiB of freed workspace
+ *    mapped between calls (GEQRF/GETRF need O(batchCount (max_m + max_n)) doubles).
  *  - Return value: 0 = enqueued; -p = host-scalar argument number p (1-based) is invalid,
  *    nothing enqueued; > 0 = a cudaError_t from the launch.
  *  - batchCount == 0 returns 0 and enqueues nothing.
