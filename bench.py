@@ -161,20 +161,31 @@ def run_oracle(arena0, off, n, ld, cores):
 
 def lapack_baseline(arena0, off, n, ld, cores, desc):
     """The paper's best CPU competitor, LAPACK dpotrf one core per matrix,
-    MKL from libtorch_cpu.so, on the oracle's sample: best of 3 (inputs restored untimed)."""
-    try:
+    MKL from libtorch_cpu.so, on the oracle's sample: best of 3 (inputs restored untimed); the
+    same with scipy's bundled OpenBLAS as `openblas` (SURVEY §8(d) secondary baseline)."""
+    def one(lib_path, kind):
         import cpu_baselines
         best, info = None, None
         for _ in range(3):
             arena = arena0.copy()
-            dt, info = cpu_baselines.dpotrf_batch(arena, off, n, ld, cores)
+            dt, info = cpu_baselines.dpotrf_batch(arena, off, n, ld, cores, lib_path=lib_path)
             best = dt if best is None else min(best, dt)
         return {"value": vbgen.expected_flops(n[info == 0]) / best / 1e9, "unit": "GFLOP/s",
-                "cores": cores, "kind": "MKL dpotrf one core per matrix" if cpu_baselines.is_mkl()
-                else "LAPACK dpotrf one core per matrix", "sample": desc.replace("OpenMP dynamic",
+                "cores": cores, "kind": kind, "sample": desc.replace("OpenMP dynamic",
                 "pthreads, LPT order,"), "seconds": best}
+    try:
+        import cpu_baselines
+        out = one(None, "MKL dpotrf one core per matrix" if cpu_baselines.is_mkl()
+                  else "LAPACK dpotrf one core per matrix")
     except Exception as e:  # a reported baseline, not the product: record why it is missing
         return {"value": None, "unavailable": str(e)[:200]}
+    try:
+        ob = cpu_baselines.openblas_path()
+        out["openblas"] = (one(ob, "OpenBLAS (scipy's bundled, LP64) dpotrf one core per matrix")
+                           if ob else {"value": None, "unavailable": "scipy's OpenBLAS not found"})
+    except Exception as e:
+        out["openblas"] = {"value": None, "unavailable": str(e)[:200]}
+    return out
 
 
 def host_cores():

@@ -62,5 +62,14 @@ def dpotrf_batch(arena: np.ndarray, offsets, n, ld, nthreads: int, lib_path: str
     return dt, info
 
 
+def openblas_path() -> str | None:
+    """scipy's bundled OpenBLAS (LP64 `scipy_dpotrf_`), the secondary CPU baseline."""
+    import glob
+    import scipy
+    libs = glob.glob(os.path.join(os.path.dirname(os.path.dirname(scipy.__file__)), "scipy.libs",
+                                  "libscipy_openblas-*.so"))
+    return libs[0] if libs else None
+
+
 def is_mkl(lib_path: str | None = None) -> bool:
     return bool(lib().lapack_batch_is_mkl((lib_path or mkl_path()).encode()))

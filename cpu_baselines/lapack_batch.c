@@ -5,7 +5,8 @@
  * cores. This file runs exactly that on the bench host: `nthreads` pthreads pull matrix
  * indices from an atomic counter (the caller passes them in LPT order) and call the LAPACK
  * `dpotrf_` resolved at run time from an already-loaded library (MKL inside libtorch_cpu.so,
- * or OpenBLAS), with MKL's per-thread thread count forced to 1 when that symbol exists.
+ * or OpenBLAS), with MKL's per-thread thread count forced to 1 when that symbol exists; scipy's
+ * bundled OpenBLAS (LP64, `scipy_dpotrf_`) with its global thread count set to 1.
  * Plain pointers, no torch types; nothing here is used by libvbatched or by the oracle.
  */
 #define _GNU_SOURCE
@@ -52,6 +53,11 @@ int lapack_batch_dpotrf(const char* lib_path, double* const* A, const int* n, co
   struct job j;
   j.potrf = (dpotrf_fn)dlsym(h, "dpotrf_");
   j.set_local = (set_local_fn)dlsym(h, "MKL_Set_Num_Threads_Local");
+  if (!j.potrf) {  // scipy's bundled OpenBLAS (LP64): prefixed symbols, a global thread count
+    j.potrf = (dpotrf_fn)dlsym(h, "scipy_dpotrf_");
+    void (*set_global)(int) = (void (*)(int))dlsym(h, "scipy_openblas_set_num_threads");
+    if (set_global) set_global(1);  /* one thread per dpotrf call; the workers give parallelism */
+  }
   if (!j.potrf) return -1;
   j.A = A;
   j.n = n;
