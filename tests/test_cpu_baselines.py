@@ -1,15 +1,12 @@
 """The bench's CPU library baselines (MKL / scipy's OpenBLAS dpotrf one core per matrix,
-cpu_baselines/) agree
-with the oracle on info and to rounding on L (it is a reported baseline, so this only checks
+cpu_baselines/) agree with the oracle on info and to rounding on L (it is a reported baseline, so this only checks
 that the number it produces comes from correct factorisations)."""
 import numpy as np
+import pytest
 
 import cpu_baselines
 import oracle
 import vbgen
-
-
-import pytest
 
 
 @pytest.mark.parametrize("which", ["mkl", "openblas"])
