@@ -53,6 +53,10 @@ namespace vb {
 #ifndef VB_PF
 #define VB_PF 0
 #endif
+// 1: the blocked kernel's ring always uses the cp.async gather path (development A/B).
+#ifndef VB_NOBULK
+#define VB_NOBULK 0
+#endif
 #ifndef VB_KREV
 #define VB_KREV 1
 #endif
@@ -117,6 +121,19 @@ VB_DEVINL unsigned long long tl_now() {
 #define TL_END(pred, v, m, kind)
 #endif
 
+
+// Optional ring-latency records (debug builds with -DVB_CHUNK_LAT, tools/chunk_lat.py): for CTAs
+// b < 64 and ring positions gi < 4096 of the blocked kernel, SM clock64() at: producer before its
+// empty-slot wait (0), after it (1), after issuing the copies (2); consumer warp 0 before its
+// full-barrier wait (3), after it (4). Same SM, so one clock domain per record.
+#ifdef VB_CHUNK_LAT
+__device__ unsigned long long* g_lat;
+#define LAT_REC(gi, slot)                                                                  \
+  if (g_lat && blockIdx.x < 64 && (gi) < 4096 && (threadIdx.x & 31) == 0)                   \
+    g_lat[((size_t)blockIdx.x * 4096 + (gi)) * 8 + (slot)] = clock64();
+#else
+#define LAT_REC(gi, slot) {}
+#endif
 
 // ---------------------------------------------------------------------------------------
 // POTF2 of an nb x nb (nb <= NM <= 32) lower block by one warp, lane r holding row r in
@@ -429,8 +446,10 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
   const int st = gi % C::STAGES;
   const uint32_t u = gi / C::STAGES;
   const int k0 = kc * C::KC;
+  LAT_REC(gi, 0)
   if (lane == 0 && u > 0) mbar_wait(&s.empty[st], (u - 1) & 1);
   __syncwarp();
+  LAT_REC(gi, 1)
   if (bulk) {
     // segments rounded up to 16 bytes: the extra rows lie inside ldda (ldda is a multiple of
     // G here) and only ever feed output rows/columns that are never stored
@@ -491,6 +510,7 @@ VB_DEVINL void issue_chunk2(Smem2<C>& s, uint32_t gi, int kc, const typename C::
     }
     cp_async_mbar_arrive_noinc(&s.full[st]);
   }
+  LAT_REC(gi, 2)
 }
 
 // TRSM of this warp's 16 rows, in registers: X = C inv(L)^T (NB = 64: two 32-column steps
@@ -589,7 +609,7 @@ VB_DEVINL void produce_matrix3(Smem2<C>& s, const typename C::E* A, int n, int l
   constexpr int NB = C::NB, MB = C::MB, KC = C::KC;
   using E = typename C::E;
   constexpr int G = C::G;
-  const bool bulk = !UP && ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && (ld % G == 0);
+  const bool bulk = !VB_NOBULK && !UP && ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && (ld % G == 0);
   const int npan = (n + NB - 1) / NB;
   int done = npan;  // panels the consumers will complete for this matrix
   fence_proxy_async();
@@ -646,7 +666,9 @@ VB_DEVINL void k_loop3(Smem2<C>& s, double (&acc)[2][C::NT][2], uint32_t& gchunk
   for (int kc = 0; kc < nk; ++kc) {
     const uint32_t gi = gchunk++;
     const int st = gi % C::STAGES;
+    if (threadIdx.x < 32) { LAT_REC(gi, 3) }
     mbar_wait(&s.full[st], (gi / C::STAGES) & 1);
+    if (threadIdx.x < 32) { LAT_REC(gi, 4) }
     if constexpr (NTL > 0) {
 #pragma unroll
       for (int kk = 0; kk < C::KC / 4; ++kk) {
@@ -1538,6 +1560,12 @@ cudaError_t launch_potrf_direct(const int* d_n, float* const* dA, const int* d_l
 }
 
 }  // namespace vb
+
+#ifdef VB_CHUNK_LAT
+extern "C" int vbatched_debug_chunk_lat(unsigned long long* dptr) {
+  return (int)cudaMemcpyToSymbol(vb::g_lat, &dptr, sizeof(dptr));
+}
+#endif
 
 #ifdef VB_TIMELINE
 extern "C" int vbatched_debug_timeline(unsigned long long* dptr) {
